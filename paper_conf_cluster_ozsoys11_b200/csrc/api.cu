@@ -1,0 +1,529 @@
+// api.cu -- the C ABI of libculzss.so (include/culzss.h) and its host
+// orchestration: parameter validation, stream-ordered workspace, the launch
+// sequence, the device error word, and the one sync that returns *out_n.
+//
+// The paper's API (PAPER.md:1@10268-10919 §III): a dynamically loaded
+// in-memory library that "gets initialized when loaded, detects GPUs, and
+// determines capabilities"; Gpu_compress() "compresses it into the given
+// memory region, and returns ... the compressed data and its length".
+
+#include <atomic>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+
+#include "../../include/culzss.h"
+#include "culzss_internal.h"
+
+namespace culzss {
+
+static std::atomic<uint64_t> g_launches{0};
+void count_launch(int k) { g_launches.fetch_add((uint64_t)k, std::memory_order_relaxed); }
+
+namespace {
+
+thread_local int t_last_cuda_error = 0;
+thread_local bool t_profiling = false;
+struct KernelTimes {
+    float chunk = -1, scan = -1, compact = -1, decode = -1, call = -1;
+};
+thread_local KernelTimes t_times;
+
+int g_device_count = -1;
+std::once_flag g_init_once;
+
+void lib_init() {
+    std::call_once(g_init_once, [] {
+        int n = 0;
+        if (cudaGetDeviceCount(&n) != cudaSuccess) {
+            n = 0;
+            cudaGetLastError();
+        }
+        g_device_count = n;
+        // keep freed workspace in the stream-ordered pool between calls
+        for (int d = 0; d < n; d++) {
+            cudaMemPool_t pool;
+            if (cudaDeviceGetDefaultMemPool(&pool, d) == cudaSuccess) {
+                uint64_t thr = UINT64_MAX;
+                cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+            }
+        }
+        cudaGetLastError();
+    });
+}
+
+struct LibLoad {
+    LibLoad() { /* device detection is lazy: CUDA may not be usable at dlopen time */ }
+} g_libload;
+
+culzss_status cuda_fail(cudaError_t e) {
+    t_last_cuda_error = (int)e;
+    return CULZSS_ERR_CUDA;
+}
+
+#define CK(expr)                                      \
+    do {                                              \
+        cudaError_t _e = (expr);                      \
+        if (_e != cudaSuccess) return cuda_fail(_e);  \
+    } while (0)
+
+culzss_status check_params(const culzss_params *p, Geometry *g) {
+    culzss_params d;
+    culzss_default_params(&d);
+    if (!p) p = &d;
+    if (p->min_match != 3 || p->chunk_size < 1 || p->window < 1 || p->window > 256 ||
+        p->max_match < 3 || p->max_match > 258 || p->reserved != 0)
+        return CULZSS_ERR_INVALID_ARG;
+    if (p->version != 0 || p->chunk_size > (uint32_t)kChunkMax || p->window > 255)
+        return CULZSS_ERR_UNSUPPORTED;
+    g->S = p->chunk_size;
+    g->W = p->window;
+    g->F = p->max_match;
+    return CULZSS_OK;
+}
+
+uint64_t n_chunks(uint64_t n, uint32_t S) { return (n + S - 1) / S; }
+
+uint64_t payload_bound(uint64_t n, uint32_t S) {
+    uint64_t full = n / S, tail = n % S;
+    uint64_t b = full * ((9ull * S + 7) / 8);
+    if (tail) b += (9 * tail + 7) / 8;
+    return b;
+}
+
+bool is_device_ptr(const void *ptr) {
+    if (!ptr) return false;
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, ptr) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+bool overlap(const void *a, size_t na, const void *b, size_t nb) {
+    uintptr_t x = (uintptr_t)a, y = (uintptr_t)b;
+    return na && nb && x < y + nb && y < x + na;
+}
+
+// Stream-ordered workspace that frees itself on scope exit.
+struct Workspace {
+    cudaStream_t st;
+    void *p = nullptr;
+    explicit Workspace(cudaStream_t s) : st(s) {}
+    cudaError_t alloc(size_t bytes) { return cudaMallocAsync(&p, bytes ? bytes : 16, st); }
+    ~Workspace() {
+        if (p) cudaFreeAsync(p, st);
+    }
+};
+
+// Pinned host word for the 8-byte D2H of a device total (one per thread).
+uint64_t *host_word() {
+    thread_local uint64_t *w = nullptr;
+    if (!w) {
+        if (cudaMallocHost(&w, 64) != cudaSuccess) {
+            cudaGetLastError();
+            w = nullptr;
+        }
+    }
+    return w;
+}
+
+// Profiling: events recorded on the call's stream at stage boundaries with
+// no intermediate host sync; elapsed times are read after the call's own
+// final synchronisation.  Stages: 0 call start, 1 after the fused chunk
+// kernel's predecessor (header), 2 after chunk, 3 after scan, 4 after
+// compact, 5 call end (after the D2H of the total).
+struct Prof {
+    static constexpr int kN = 6;
+    cudaEvent_t e[kN] = {};
+    bool used[kN] = {};
+    bool ready = false;
+    void rec(int i, cudaStream_t st) {
+        if (!t_profiling) return;
+        if (!ready) {
+            for (auto &x : e) cudaEventCreate(&x);
+            ready = true;
+        }
+        cudaEventRecord(e[i], st);
+        used[i] = true;
+    }
+    float between(int a, int b) {
+        float v = -1;
+        if (ready && used[a] && used[b] && cudaEventElapsedTime(&v, e[a], e[b]) != cudaSuccess) {
+            cudaGetLastError();
+            v = -1;
+        }
+        return v;
+    }
+    void reset() {
+        for (auto &u : used) u = false;
+    }
+};
+thread_local Prof t_prof;
+
+void prof_finish_compress() {
+    if (!t_profiling) return;
+    t_times.chunk = t_prof.between(1, 2);
+    t_times.scan = t_prof.between(2, 3);
+    t_times.compact = t_prof.between(3, 4);
+    t_times.call = t_prof.between(0, 5);
+}
+
+// Core compression of n bytes at device `in` into: payload region `pay`
+// (capacity checked by callers), table `table` (may be null), total payload
+// bytes -> device word `dev_total`.  Sizes go to `sizes` (device, C words).
+culzss_status compress_core(const uint8_t *in, uint64_t n, const Geometry &g, uint8_t *pay,
+                            uint32_t *table, uint32_t *sizes_out, uint64_t *dev_total,
+                            cudaStream_t st) {
+    const uint64_t C = n_chunks(n, g.S);
+    const uint64_t stride = bucket_stride(g.S);
+    const uint64_t scan_ws = scan_workspace_words(C);
+    // workspace: bucket | sizes | offsets | scan ws
+    const uint64_t bucket_bytes = C * stride + 16;
+    const uint64_t sizes_off = (bucket_bytes + 255) / 256 * 256;
+    const uint64_t offs_off = sizes_off + (C * 4 + 255) / 256 * 256;
+    const uint64_t ws_off = offs_off + (C * 8 + 255) / 256 * 256;
+    const uint64_t total_bytes = ws_off + scan_ws * 8;
+    Workspace ws(st);
+    CK(ws.alloc(total_bytes));
+    uint8_t *base = static_cast<uint8_t *>(ws.p);
+    uint8_t *bucket = base;
+    uint32_t *sizes = sizes_out ? sizes_out : reinterpret_cast<uint32_t *>(base + sizes_off);
+    uint64_t *offsets = reinterpret_cast<uint64_t *>(base + offs_off);
+    uint64_t *scanws = reinterpret_cast<uint64_t *>(base + ws_off);
+
+    t_prof.rec(1, st);
+    CK(launch_chunk_kernel(kModeCompress, in, n, g, bucket, sizes, nullptr, st));
+    t_prof.rec(2, st);
+    CK(launch_scan(sizes, C, offsets, dev_total, scanws, st));
+    t_prof.rec(3, st);
+    CK(launch_compact(bucket, stride, sizes, offsets, C, pay, table, st));
+    t_prof.rec(4, st);
+    return CULZSS_OK;
+}
+
+}  // namespace
+}  // namespace culzss
+
+using namespace culzss;
+
+extern "C" {
+
+void culzss_default_params(culzss_params *p) {
+    if (!p) return;
+    p->chunk_size = 4096;
+    p->window = 128;
+    p->max_match = 128;
+    p->min_match = 3;
+    p->version = 0;
+    p->reserved = 0;
+}
+
+size_t culzss_max_compressed_size(size_t n, const culzss_params *p) {
+    culzss_params d;
+    culzss_default_params(&d);
+    if (!p) p = &d;
+    if (p->chunk_size < 1) return 0;
+    uint64_t C = n_chunks(n, p->chunk_size);
+    return (size_t)(32 + 4 * C + payload_bound(n, p->chunk_size));
+}
+
+int culzss_device_count(void) {
+    lib_init();
+    return g_device_count;
+}
+
+uint64_t culzss_launch_count(void) { return g_launches.load(); }
+
+void culzss_set_profiling(int enable) { t_profiling = enable != 0; }
+
+float culzss_last_kernel_ms(const char *name) {
+    if (!name) return -1;
+    if (!strcmp(name, "chunk")) return t_times.chunk;
+    if (!strcmp(name, "scan")) return t_times.scan;
+    if (!strcmp(name, "compact")) return t_times.compact;
+    if (!strcmp(name, "decode")) return t_times.decode;
+    if (!strcmp(name, "call")) return t_times.call;
+    return -1;
+}
+
+const char *culzss_status_string(culzss_status s) {
+    switch (s) {
+        case CULZSS_OK: return "ok";
+        case CULZSS_ERR_INVALID_ARG: return "invalid argument";
+        case CULZSS_ERR_UNSUPPORTED: return "unsupported parameters";
+        case CULZSS_ERR_BUFFER_TOO_SMALL: return "buffer too small";
+        case CULZSS_ERR_CORRUPT: return "corrupt stream";
+        case CULZSS_ERR_CUDA: return "CUDA error";
+        case CULZSS_ERR_NO_DEVICE: return "no CUDA device";
+    }
+    return "unknown status";
+}
+
+int culzss_last_cuda_error(void) { return t_last_cuda_error; }
+
+culzss_status culzss_write_header(void *out, size_t n_total, const culzss_params *p,
+                                  culzss_stream_t stream) {
+    lib_init();
+    if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
+    Geometry g;
+    culzss_status s = check_params(p, &g);
+    if (s != CULZSS_OK) return s;
+    if (!is_device_ptr(out)) return CULZSS_ERR_INVALID_ARG;
+    if (n_chunks(n_total, g.S) > 0xFFFFFFFFull) return CULZSS_ERR_INVALID_ARG;
+    cudaError_t e = launch_header(static_cast<uint8_t *>(out), n_total, g, (cudaStream_t)stream);
+    return e == cudaSuccess ? CULZSS_OK : cuda_fail(e);
+}
+
+culzss_status culzss_compress(const void *in, size_t n, void *out, size_t *out_n,
+                              const culzss_params *p, culzss_stream_t stream) {
+    lib_init();
+    if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
+    if (!out_n) return CULZSS_ERR_INVALID_ARG;
+    Geometry g;
+    culzss_status s = check_params(p, &g);
+    if (s != CULZSS_OK) return s;
+    const uint64_t C = n_chunks(n, g.S);
+    if (C > 0xFFFFFFFFull) return CULZSS_ERR_INVALID_ARG;
+    const uint64_t bound = 32 + 4 * C + payload_bound(n, g.S);
+    if (*out_n < bound) {
+        *out_n = (size_t)bound;
+        return CULZSS_ERR_BUFFER_TOO_SMALL;
+    }
+    if (!is_device_ptr(out) || (n && !is_device_ptr(in))) return CULZSS_ERR_INVALID_ARG;
+    if (overlap(in, n, out, bound)) return CULZSS_ERR_INVALID_ARG;
+    cudaStream_t st = (cudaStream_t)stream;
+    uint8_t *o = static_cast<uint8_t *>(out);
+    uint64_t *hw = host_word();
+    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
+    t_prof.reset();
+    t_prof.rec(0, st);
+    {
+        cudaError_t e = launch_header(o, n, g, st);
+        if (e != cudaSuccess) return cuda_fail(e);
+    }
+    if (n == 0) {
+        CK(cudaStreamSynchronize(st));
+        *out_n = 32;
+        return CULZSS_OK;
+    }
+    uint64_t *dev_total = nullptr;
+    CK(cudaMallocAsync(&dev_total, 8, st));
+    s = compress_core(static_cast<const uint8_t *>(in), n, g, o + 32 + 4 * C,
+                      reinterpret_cast<uint32_t *>(o + 32), nullptr, dev_total, st);
+    if (s == CULZSS_OK) {
+        cudaError_t e = cudaMemcpyAsync(hw, dev_total, 8, cudaMemcpyDeviceToHost, st);
+        t_prof.rec(5, st);
+        if (e == cudaSuccess) e = cudaFreeAsync(dev_total, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+        if (e != cudaSuccess) return cuda_fail(e);
+        prof_finish_compress();
+        *out_n = (size_t)(32 + 4 * C + *hw);
+        return CULZSS_OK;
+    }
+    cudaFreeAsync(dev_total, st);
+    return s;
+}
+
+culzss_status culzss_compress_chunks(const void *in_slice, size_t slice_n, void *payload,
+                                     size_t *payload_n, uint32_t *chunk_sizes,
+                                     const culzss_params *p, culzss_stream_t stream) {
+    lib_init();
+    if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
+    if (!payload_n) return CULZSS_ERR_INVALID_ARG;
+    Geometry g;
+    culzss_status s = check_params(p, &g);
+    if (s != CULZSS_OK) return s;
+    const uint64_t bound = payload_bound(slice_n, g.S);
+    if (*payload_n < bound) {
+        *payload_n = (size_t)bound;
+        return CULZSS_ERR_BUFFER_TOO_SMALL;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    if (slice_n == 0) {
+        *payload_n = 0;
+        return CULZSS_OK;
+    }
+    if (!is_device_ptr(in_slice) || !is_device_ptr(payload) || !is_device_ptr(chunk_sizes))
+        return CULZSS_ERR_INVALID_ARG;
+    uint64_t *hw = host_word();
+    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
+    uint64_t *dev_total = nullptr;
+    t_prof.reset();
+    t_prof.rec(0, st);
+    CK(cudaMallocAsync(&dev_total, 8, st));
+    s = compress_core(static_cast<const uint8_t *>(in_slice), slice_n, g,
+                      static_cast<uint8_t *>(payload), nullptr, chunk_sizes, dev_total, st);
+    if (s == CULZSS_OK) {
+        cudaError_t e = cudaMemcpyAsync(hw, dev_total, 8, cudaMemcpyDeviceToHost, st);
+        t_prof.rec(5, st);
+        if (e == cudaSuccess) e = cudaFreeAsync(dev_total, st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+        if (e != cudaSuccess) return cuda_fail(e);
+        prof_finish_compress();
+        *payload_n = (size_t)*hw;
+        return CULZSS_OK;
+    }
+    cudaFreeAsync(dev_total, st);
+    return s;
+}
+
+culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host, size_t *out_n,
+                                   const culzss_params *p, culzss_stream_t stream) {
+    lib_init();
+    if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
+    if (!out_n || (n && !in_host) || !out_host) return CULZSS_ERR_INVALID_ARG;
+    Geometry g;
+    culzss_status s = check_params(p, &g);
+    if (s != CULZSS_OK) return s;
+    const uint64_t C = n_chunks(n, g.S);
+    const uint64_t bound = 32 + 4 * C + payload_bound(n, g.S);
+    if (*out_n < bound) {
+        *out_n = (size_t)bound;
+        return CULZSS_ERR_BUFFER_TOO_SMALL;
+    }
+    cudaStream_t st = (cudaStream_t)stream;
+    Workspace ws(st);
+    const uint64_t in_bytes = (n + 255) / 256 * 256;
+    CK(ws.alloc(in_bytes + bound));
+    uint8_t *din = static_cast<uint8_t *>(ws.p);
+    uint8_t *dout = din + in_bytes;
+    if (n) CK(cudaMemcpyAsync(din, in_host, n, cudaMemcpyHostToDevice, st));
+    size_t on = (size_t)bound;
+    s = culzss_compress(din, n, dout, &on, p, stream);
+    if (s != CULZSS_OK) return s;
+    CK(cudaMemcpyAsync(out_host, dout, on, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    *out_n = on;
+    return CULZSS_OK;
+}
+
+static culzss_status read_header(const void *in, size_t in_n, Geometry *g, uint64_t *n,
+                                 uint64_t *C, cudaStream_t st) {
+    if (in_n < 32) return CULZSS_ERR_CORRUPT;
+    uint64_t *hw = host_word();
+    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
+    uint8_t *h = reinterpret_cast<uint8_t *>(hw);
+    CK(cudaMemcpyAsync(h, in, 32, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    auto le = [&](int off, int nb) {
+        uint64_t v = 0;
+        for (int i = 0; i < nb; i++) v |= (uint64_t)h[off + i] << (8 * i);
+        return v;
+    };
+    if (h[0] != 'C' || h[1] != 'L' || h[2] != 'Z' || h[3] != 'S') return CULZSS_ERR_CORRUPT;
+    if (le(4, 2) != 1 || le(6, 2) != 32 || h[29] || h[30] || h[31]) return CULZSS_ERR_CORRUPT;
+    culzss_params p;
+    p.chunk_size = (uint32_t)le(8, 4);
+    p.window = (uint16_t)le(24, 2);
+    p.max_match = (uint16_t)le(26, 2);
+    p.min_match = h[28];
+    p.version = 0;
+    p.reserved = 0;
+    if (p.min_match != 3 || p.chunk_size < 1 || p.window < 1 || p.window > 256 ||
+        p.max_match < 3 || p.max_match > 258)
+        return CULZSS_ERR_CORRUPT;
+    *n = le(16, 8);
+    *C = le(12, 4);
+    if (*C != n_chunks(*n, p.chunk_size)) return CULZSS_ERR_CORRUPT;
+    culzss_status s = check_params(&p, g);
+    return s == CULZSS_OK ? CULZSS_OK : CULZSS_ERR_UNSUPPORTED;
+}
+
+culzss_status culzss_decompressed_size(const void *in, size_t in_n, size_t *n,
+                                       culzss_stream_t stream) {
+    lib_init();
+    if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
+    if (!n || !is_device_ptr(in)) return CULZSS_ERR_INVALID_ARG;
+    Geometry g;
+    uint64_t nn, C;
+    culzss_status s = read_header(in, in_n, &g, &nn, &C, (cudaStream_t)stream);
+    if (s == CULZSS_OK || s == CULZSS_ERR_UNSUPPORTED) *n = (size_t)nn;
+    return s == CULZSS_ERR_UNSUPPORTED ? CULZSS_OK : s;
+}
+
+culzss_status culzss_decompress(const void *in, size_t in_n, void *out, size_t *out_n,
+                                const culzss_params *, culzss_stream_t stream) {
+    lib_init();
+    if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
+    if (!out_n || !is_device_ptr(in)) return CULZSS_ERR_INVALID_ARG;
+    cudaStream_t st = (cudaStream_t)stream;
+    Geometry g;
+    uint64_t n, C;
+    culzss_status s = read_header(in, in_n, &g, &n, &C, st);
+    if (s != CULZSS_OK) return s;
+    if (in_n < 32 + 4 * C) return CULZSS_ERR_CORRUPT;
+    if (*out_n < n) {
+        *out_n = (size_t)n;
+        return CULZSS_ERR_BUFFER_TOO_SMALL;
+    }
+    if (n == 0) {
+        if (in_n != 32) return CULZSS_ERR_CORRUPT;
+        *out_n = 0;
+        return CULZSS_OK;
+    }
+    if (!is_device_ptr(out) || overlap(in, in_n, out, n)) return CULZSS_ERR_INVALID_ARG;
+    // workspace: aligned copy of the table | offsets | scan ws | total | err
+    const uint64_t tab_off = 0;
+    const uint64_t offs_off = (C * 4 + 255) / 256 * 256;
+    const uint64_t ws_off = offs_off + (C * 8 + 255) / 256 * 256;
+    const uint64_t tot_off = ws_off + (scan_workspace_words(C) * 8 + 255) / 256 * 256;
+    Workspace ws(st);
+    CK(ws.alloc(tot_off + 256));
+    uint8_t *base = static_cast<uint8_t *>(ws.p);
+    uint32_t *sizes = reinterpret_cast<uint32_t *>(base + tab_off);
+    uint64_t *offsets = reinterpret_cast<uint64_t *>(base + offs_off);
+    uint64_t *scanws = reinterpret_cast<uint64_t *>(base + ws_off);
+    uint64_t *total = reinterpret_cast<uint64_t *>(base + tot_off);
+    uint32_t *err = reinterpret_cast<uint32_t *>(base + tot_off + 8);
+    const uint8_t *src = static_cast<const uint8_t *>(in);
+    CK(cudaMemcpyAsync(sizes, src + 32, C * 4, cudaMemcpyDeviceToDevice, st));
+    CK(cudaMemsetAsync(err, 0, 4, st));
+    CK(launch_scan(sizes, C, offsets, total, scanws, st));
+    uint64_t *hw = host_word();
+    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
+    CK(cudaMemcpyAsync(hw, total, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (32 + 4 * C + hw[0] != in_n) return CULZSS_ERR_CORRUPT;
+    t_prof.reset();
+    t_prof.rec(1, st);
+    CK(launch_decode(src + 32 + 4 * C, sizes, offsets, C, n, g, static_cast<uint8_t *>(out),
+                     err, st));
+    t_prof.rec(2, st);
+    CK(cudaMemcpyAsync(hw, err, 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (t_profiling) t_times.decode = t_prof.between(1, 2);
+    if (reinterpret_cast<uint32_t *>(hw)[0]) return CULZSS_ERR_CORRUPT;
+    *out_n = (size_t)n;
+    return CULZSS_OK;
+}
+
+static culzss_status debug_entry(int mode, const void *in, size_t n, void *dst,
+                                 const culzss_params *p, culzss_stream_t stream) {
+    lib_init();
+    if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
+    Geometry g;
+    culzss_status s = check_params(p, &g);
+    if (s != CULZSS_OK) return s;
+    if (mode == kModeDumpMatch && g.F > 255) return CULZSS_ERR_UNSUPPORTED;
+    if (n == 0) return CULZSS_OK;
+    if (!is_device_ptr(in) || !is_device_ptr(dst)) return CULZSS_ERR_INVALID_ARG;
+    cudaStream_t st = (cudaStream_t)stream;
+    CK(launch_chunk_kernel(mode, static_cast<const uint8_t *>(in), n, g, nullptr, nullptr, dst, st));
+    CK(cudaStreamSynchronize(st));
+    return CULZSS_OK;
+}
+
+culzss_status culzss_match_search(const void *in, size_t n, uint8_t *LD, const culzss_params *p,
+                                  culzss_stream_t stream) {
+    return debug_entry(kModeDumpMatch, in, n, LD, p, stream);
+}
+
+culzss_status culzss_parse_tokens(const void *in, size_t n, uint32_t *tok, const culzss_params *p,
+                                  culzss_stream_t stream) {
+    return debug_entry(kModeDumpTokens, in, n, tok, p, stream);
+}
+
+}  // extern "C"

@@ -1,0 +1,296 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Bit-exact for every byte of the stream (integer work), per-position (L, D)
+for the match search, per-position tokens for the greedy parse, and exact
+round trips for the decoder.  Inputs come from the seeded generators; no
+expected value comes from the CUDA path.
+"""
+import struct
+
+import numpy as np
+import pytest
+
+import oracle as O
+from paper_conf_cluster_ozsoys11_b200 import datagen
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def env():
+    import torch
+    from paper_conf_cluster_ozsoys11_b200 import build, culzss
+    build.build()
+    assert culzss.device_count() >= 1
+    return torch, culzss
+
+
+def dev(torch, a):
+    a = np.ascontiguousarray(a, dtype=np.uint8)
+    return torch.from_numpy(a.copy()).cuda() if a.size else torch.empty(0, dtype=torch.uint8, device="cuda")
+
+
+def gpu_stream(env, x, **kw):
+    torch, culzss = env
+    p = culzss.Params.make(**kw) if kw else None
+    return culzss.compress(dev(torch, x), p).cpu().numpy().tobytes()
+
+
+def adversarial_inputs():
+    rng = np.random.default_rng(123)
+    cases = {
+        "empty": np.zeros(0, np.uint8),
+        "one": np.array([7], np.uint8),
+        "zeros_64k": np.zeros(65536, np.uint8),
+        "ff_5000": np.full(5000, 255, np.uint8),
+        "ramp": (np.arange(10000) & 0xFF).astype(np.uint8),
+        "random_100k": rng.integers(0, 256, 100000, dtype=np.uint8),
+        "binary_30k": rng.integers(0, 2, 30000, dtype=np.uint8),
+        "ternary_30k": rng.integers(0, 3, 30000, dtype=np.uint8),
+        "figure1": np.frombuffer(b"I meant what I said\nand I said what I meant\n\nFrom there to here\n"
+                                 b"from here to there\nI said what I meant", np.uint8),
+    }
+    for d in list(range(1, 20)) + [31, 32, 33, 63, 64, 65, 100, 126, 127, 128, 129, 130, 200, 255, 256]:
+        base = rng.integers(0, 256, d, dtype=np.uint8)
+        cases[f"period{d}"] = np.tile(base, 9000 // d + 1)[:9000 + d]
+    runs = np.repeat(rng.integers(0, 4, 3000, dtype=np.uint8), rng.integers(1, 300, 3000))
+    cases["runs_mixed"] = runs[:200000]
+    return cases
+
+
+@pytest.mark.parametrize("name", list(adversarial_inputs().keys()))
+def test_stream_bit_exact_adversarial(env, name):
+    x = adversarial_inputs()[name]
+    assert gpu_stream(env, x) == O.compress(x)
+
+
+@pytest.mark.parametrize("n", [1, 2, 3, 4, 5, 127, 128, 129, 4093, 4095, 4096, 4097, 8191, 8192, 8195,
+                               (1 << 20) + 13])
+@pytest.mark.parametrize("kind", ["english", "random", "runs20"])
+def test_stream_bit_exact_sizes(env, n, kind):
+    x = datagen.generate(kind, n, seed=n)
+    assert gpu_stream(env, x) == O.compress(x)
+
+
+@pytest.mark.parametrize("kind", datagen.GENERATORS)
+def test_stream_bit_exact_generators(env, kind):
+    x = datagen.generate(kind, (1 << 20) + 777, seed=5)
+    assert gpu_stream(env, x) == O.compress(x)
+
+
+def test_config1_english_64k_bit_exact(env):
+    """BASELINE configs[0]: 64 KB English-like text, paper params, full stream."""
+    for kind in ("english", "wordlist"):
+        x = datagen.generate(kind, 64 << 10, seed=1)
+        assert gpu_stream(env, x) == O.compress(x)
+
+
+@pytest.mark.parametrize("S,W,F", [(4096, 1, 3), (4096, 2, 4), (4096, 16, 18), (4096, 64, 200),
+                                   (4096, 255, 258), (4096, 128, 129), (1, 128, 128), (2, 128, 128),
+                                   (100, 7, 9), (128, 128, 128), (1000, 128, 128), (4000, 100, 250),
+                                   (129, 3, 5)])
+def test_stream_params_variants(env, S, W, F):
+    for kind in ("english", "runs20", "period20", "binary"):
+        if kind == "binary":
+            x = np.random.default_rng(S + W + F).integers(0, 2, 50000, dtype=np.uint8)
+        else:
+            x = datagen.generate(kind, 50000, seed=S)
+        assert gpu_stream(env, x, S=S, W=W, F=F) == O.compress(x, S=S, W=W, F=F), kind
+
+
+@pytest.mark.parametrize("kind", ["english", "csource", "runs20", "period20", "random", "tarmix"])
+def test_match_search_per_position(env, kind):
+    """Row a2: (L, D) at every position of several chunks + a ragged tail."""
+    torch, culzss = env
+    x = datagen.generate(kind, 5 * 4096 + 1234, seed=9)
+    L, D = culzss.match_search(dev(torch, x))
+    L, D = L.cpu().numpy(), D.cpu().numpy()
+    for c in range(6):
+        chunk = x[c * 4096:(c + 1) * 4096]
+        eL, eD = O.match_all(chunk)
+        np.testing.assert_array_equal(L[c * 4096:c * 4096 + chunk.size], eL)
+        np.testing.assert_array_equal(D[c * 4096:c * 4096 + chunk.size], eD)
+
+
+@pytest.mark.parametrize("W,F", [(128, 128), (5, 7), (255, 255), (1, 3)])
+def test_match_search_adversarial(env, W, F):
+    torch, culzss = env
+    for name, x in adversarial_inputs().items():
+        x = x[:3 * 4096 + 5]
+        if x.size == 0:
+            continue
+        L, D = culzss.match_search(dev(torch, x), culzss.Params.make(W=W, F=F))
+        L, D = L.cpu().numpy(), D.cpu().numpy()
+        for c in range((x.size + 4095) // 4096):
+            chunk = x[c * 4096:(c + 1) * 4096]
+            eL, eD = O.match_all(chunk, W=W, F=F)
+            np.testing.assert_array_equal(L[c * 4096:c * 4096 + chunk.size], eL, err_msg=name)
+            np.testing.assert_array_equal(D[c * 4096:c * 4096 + chunk.size], eD, err_msg=name)
+
+
+def expand_tokens(toks, m):
+    out = np.zeros(m, np.int64)
+    p = 0
+    for t in toks:
+        if t[0] == "L":
+            out[p] = 1
+            p += 1
+        else:
+            out[p] = (t[2] << 16) | t[1]
+            p += t[2]
+    assert p == m
+    return out
+
+
+@pytest.mark.parametrize("kind", ["english", "csource", "runs20", "period20", "random", "tarmix",
+                                  "wordlist"])
+def test_parse_tokens(env, kind):
+    """Row a3: the speculative segment-parallel parse equals the serial greedy parse."""
+    torch, culzss = env
+    x = datagen.generate(kind, 4 * 4096 + 3000, seed=3)
+    tok = culzss.parse_tokens(dev(torch, x)).cpu().numpy().astype(np.int64) & 0xFFFFFFFF
+    for c in range(5):
+        chunk = x[c * 4096:(c + 1) * 4096]
+        np.testing.assert_array_equal(tok[c * 4096:c * 4096 + chunk.size],
+                                      expand_tokens(O.tokens_chunk(chunk), chunk.size))
+
+
+@pytest.mark.parametrize("kind", datagen.GENERATORS)
+def test_roundtrip_device(env, kind):
+    torch, culzss = env
+    x = dev(torch, datagen.generate(kind, 3 * (1 << 20) + 99, seed=2))
+    s = culzss.compress(x)
+    y = culzss.decompress(s)
+    assert torch.equal(x, y)
+
+
+def test_gpu_decoder_reads_oracle_streams(env):
+    torch, culzss = env
+    for name, x in adversarial_inputs().items():
+        s = O.compress(x)
+        y = culzss.decompress(dev(torch, np.frombuffer(s, np.uint8)))
+        assert y.cpu().numpy().tobytes() == x.tobytes(), name
+
+
+def test_gpu_decoder_rejects_corrupt(env):
+    """Same malformations as the oracle pins (tests/test_oracle_pins.py)."""
+    torch, culzss = env
+    import test_oracle_pins as P
+    for _, s in P.CORRUPT_STREAMS:
+        st, _ = culzss.decompress_status(dev(torch, np.frombuffer(s, np.uint8)))
+        assert st == culzss.ERR_CORRUPT, s
+    # random mutations: CORRUPT or same answer as the oracle decoder
+    rng = np.random.default_rng(5)
+    x = datagen.generate("english", 20000, seed=4)
+    base = bytearray(O.compress(x))
+    for _ in range(200):
+        s = bytearray(base)
+        for _ in range(int(rng.integers(1, 4))):
+            i = int(rng.integers(0, len(s)))
+            s[i] ^= int(rng.integers(1, 256))
+        ost, oout = O.decompress_status(bytes(s))
+        gst, gout = culzss.decompress_status(dev(torch, np.frombuffer(bytes(s), np.uint8)))
+        if ost == O.OK:
+            assert gst == culzss.OK and gout.cpu().numpy().tobytes() == oout
+        else:
+            assert gst in (culzss.ERR_CORRUPT, culzss.ERR_UNSUPPORTED)
+
+
+def test_unaligned_input_and_output(env):
+    torch, culzss = env
+    x = datagen.generate("csource", 100000, seed=8)
+    buf = dev(torch, x)
+    out = torch.zeros(culzss.max_compressed_size(90000) + 16, dtype=torch.uint8, device="cuda")
+    for off in (1, 2, 3, 5, 15):
+        expect = O.compress(x[off:off + 90000])
+        for oo in (0, 1, 3):
+            n = culzss.compress_into(buf[off:off + 90000], out[oo:])
+            assert out[oo:oo + n].cpu().numpy().tobytes() == expect, (off, oo)
+
+
+def test_buffer_too_small_and_invalid(env):
+    torch, culzss = env
+    x = dev(torch, datagen.generate("english", 10000, seed=1))
+    out = torch.empty(100, dtype=torch.uint8, device="cuda")
+    with pytest.raises(culzss.CulzssError) as e:
+        culzss.compress_into(x, out)
+    assert e.value.status == culzss.ERR_BUFFER_TOO_SMALL
+    with pytest.raises(culzss.CulzssError) as e:
+        culzss.compress(x, culzss.Params.make(MIN=2))
+    assert e.value.status == culzss.ERR_INVALID_ARG
+    with pytest.raises(culzss.CulzssError) as e:
+        culzss.compress(x, culzss.Params.make(S=8192))
+    assert e.value.status == culzss.ERR_UNSUPPORTED
+
+
+def test_compress_host_matches(env):
+    torch, culzss = env
+    x = datagen.generate("tarmix", 300000, seed=6)
+    assert culzss.compress_host(x).tobytes() == O.compress(x)
+    assert culzss.compress_host(x[:0]).tobytes() == O.compress(x[:0])
+
+
+def test_sharded_assembly_equals_single(env):
+    """SURVEY §8(e) on one GPU: R simulated ranks compress chunk ranges with
+    culzss_compress_chunks; placing table slices at 32 + 4*c0 and payloads
+    at 32 + 4C + sum of earlier totals reproduces the 1-call stream."""
+    torch, culzss = env
+    x_np = datagen.generate("csource", 37 * 4096 + 1111, seed=12)
+    x = dev(torch, x_np)
+    ref = culzss.compress(x).cpu().numpy().tobytes()
+    assert ref == O.compress(x_np)
+    n, S = x_np.size, 4096
+    C = (n + S - 1) // S
+    for R in (2, 3, 4, 8):
+        parts, totals, tables = [], [], []
+        for r in range(R):
+            c0, c1 = r * C // R, (r + 1) * C // R
+            sl = x[c0 * S:min(c1 * S, n)]
+            pay = torch.empty(max(1, culzss.max_compressed_size(sl.numel()) - 32), dtype=torch.uint8, device="cuda")
+            sizes = torch.zeros(max(1, c1 - c0), dtype=torch.int32, device="cuda")
+            t = culzss.compress_chunks(sl, pay, sizes)
+            parts.append(pay[:t])
+            totals.append(t)
+            tables.append(sizes[:c1 - c0])
+        out = torch.empty(32 + 4 * C + sum(totals), dtype=torch.uint8, device="cuda")
+        culzss.write_header(out, n)
+        out[32:32 + 4 * C] = torch.cat(tables).view(torch.uint8)
+        pos = 32 + 4 * C
+        for r in range(R):
+            out[pos:pos + totals[r]] = parts[r]
+            pos += totals[r]
+        assert out.cpu().numpy().tobytes() == ref, R
+
+
+# ------------------------------------------------------------ full-size configs
+def _sampled_chunk_check(x_np, stream: bytes, nsample: int, seed: int):
+    n, S = x_np.size, 4096
+    C = (n + S - 1) // S
+    hdr = struct.unpack("<4sHHIIQHHB3x", stream[:32])
+    assert hdr == (b"CLZS", 1, 32, S, C, n, 128, 128, 3)
+    sizes = np.frombuffer(stream, dtype="<u4", count=C, offset=32).astype(np.int64)
+    offs = 32 + 4 * C + np.concatenate([[0], np.cumsum(sizes)])
+    assert offs[-1] == len(stream)
+    rng = np.random.default_rng(seed)
+    picks = set(rng.integers(0, C, nsample).tolist()) | {0, C - 1}
+    for c in sorted(picks):
+        chunk = x_np[c * S:(c + 1) * S]
+        assert stream[offs[c]:offs[c + 1]] == O.compress_chunk(chunk), c
+
+
+@pytest.mark.parametrize("cfg", ["c2_csource_128m", "c3_runs20_1g", "c4_random_1g"])
+def test_full_size_configs(env, cfg):
+    """BASELINE configs at full size, in the launch configuration bench.py
+    times: header, table sum, >=512 oracle-checked chunks (+ first/last), and
+    an exact on-device round trip of the whole input."""
+    torch, culzss = env
+    spec = datagen.CONFIGS[cfg]
+    x_np = datagen.generate(spec["kind"], spec["n"], spec["seed"])
+    x = torch.from_numpy(x_np).cuda()
+    s = culzss.compress(x)
+    stream = s.cpu().numpy().tobytes()
+    _sampled_chunk_check(x_np, stream, 512, seed=len(stream))
+    y = culzss.decompress(s)
+    assert torch.equal(x, y)
+    del y, s, x
+    torch.cuda.empty_cache()

@@ -223,7 +223,7 @@ def _stream(n, payload_bits, S=4096):
     return header(n, S) + struct.pack("<I", len(payload)) + payload
 
 
-@pytest.mark.parametrize("name,stream", [
+CORRUPT_STREAMS = [
     ("bad magic", b"CLZX" + _stream(4, lit("a") + mat(1, 3))[4:]),
     ("d > produced", _stream(4, lit("a") + mat(2, 3))),
     ("L > remaining", _stream(3, lit("a") + mat(1, 3))),
@@ -236,7 +236,10 @@ def _stream(n, payload_bits, S=4096):
     ("reserved", _stream(1, lit("a"))[:29] + b"\x01\x00\x00" + _stream(1, lit("a"))[32:]),
     ("bad params", struct.pack("<4sHHIIQHHB3x", b"CLZS", 1, 32, 4096, 1, 1, 0, 128, 3)
      + struct.pack("<I", 2) + bits_to_bytes(lit("a"))),
-])
+]
+
+
+@pytest.mark.parametrize("name,stream", CORRUPT_STREAMS)
 def test_decoder_rejects_corrupt(name, stream):
     st, _ = O.decompress_status(stream)
     assert st == O.ERR_CORRUPT, name
