@@ -1,0 +1,370 @@
+#!/usr/bin/env python
+"""Benchmark: chunked LZSS compression throughput on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2_csource_128m]
+    python bench.py --impl reference ...        # the CPU oracle as the reference arm
+    torchrun --nproc-per-node N bench.py --gpus N ...
+
+One step = one pass of the whole hot path over the
+rank's input, resident in HBM: culzss_compress at N = 1; at N > 1 each rank
+compresses its contiguous chunk range with culzss_compress_chunks and the
+ranks allgather their compressed totals over NCCL (the one exchange step;
+weak scaling: every rank holds one config-sized slice).  Timing is device
+time from CUDA events recorded by the library on the call's stream (the
+whole call, including the 8-byte D2H of the total); L2 is flushed between
+steps; the max over ranks is reported.  Rank 0 prints one JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_cluster_ozsoys11_b200 import datagen  # noqa: E402
+
+METRIC = "LZSS compress GB/s (input) at 1/2/4/8 B200 + ratio, vs CPU oracle"
+UNIT = "GB/s"
+PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FALLBACK_HBM = 6650.0  # B200_PROFILING.md fallback
+CONFIG_TEXT = {
+    "c1_english_64k": "64 KiB English-like text (english generator, seed 1)",
+    "c2_csource_128m": "128 MiB source-code-like text (csource generator, seed 2; PAPER.md:1@23843 'C files')",
+    "c3_runs20_1g": "1 GiB runs of 20 identical bytes (runs20 generator, seed 3; PAPER.md:1@24662)",
+    "c4_random_1g": "1 GiB random bytes (splitmix64, seed 4)",
+    "c5_tarmix_64g": "64 GiB tarball-like mix (tarmix generator, seed 5) -- per-rank slices",
+}
+
+
+def parse_args():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["culzss", "reference"], default="culzss")
+    ap.add_argument("--config", default="c2_csource_128m", choices=sorted(datagen.CONFIGS))
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    return ap.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def rank_input(cfg: str, rank: int, world: int) -> np.ndarray:
+    """Per-rank slice: rank 0 of N=1 holds exactly the config input; for N > 1
+    each rank holds one config-sized, chunk-aligned slice of an N-times larger
+    input (seed offset by rank), except c5 whose 64 GiB is split N ways."""
+    spec = datagen.CONFIGS[cfg]
+    n = spec["n"]
+    if cfg == "c5_tarmix_64g":
+        n = n // world
+    seed = spec["seed"] + 1000 * rank
+    return datagen.generate(spec["kind"], n, seed)
+
+
+def load_peaks():
+    try:
+        p = json.load(open(PEAKS_PATH))
+        return float(p["hbm_gbs"]), float(p.get("sm_max_mhz", 1965.0)), "measured"
+    except Exception:
+        return FALLBACK_HBM, 1965.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.proc = None
+        self.gpu = gpu_index
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100", "-i", str(self.gpu)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL,
+                text=True)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            out, _ = self.proc.communicate(timeout=5)
+        except Exception:
+            self.proc.kill()
+            out = ""
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                smax.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[3:7]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cpu_baseline(x: np.ndarray, stream_bytes: bytes | None, budget_s: float = 10.0):
+    """The C oracle, as it stands, on the host cores over a bounded sample:
+    contiguous chunk ranges in threads (ctypes releases the GIL), the paper's
+    Pthread decomposition (PAPER.md:1@11659).  The sample is the config
+    input's leading chunks, sized from a 1-chunk-per-thread probe to about
+    budget_s of wall time."""
+    import concurrent.futures as cf
+    import oracle
+    S = 4096
+    cores = max(1, min(len(os.sched_getaffinity(0)), 64))
+    C = (x.size + S - 1) // S
+    t0 = time.perf_counter()
+    oracle.compress_range(x, 0, min(C, 16))
+    per_chunk = (time.perf_counter() - t0) / min(C, 16)
+    nchunks = int(min(C, max(cores, budget_s * cores / max(per_chunk, 1e-6))))
+    nchunks = max(1, nchunks)
+    bounds = [(i * nchunks // cores, (i + 1) * nchunks // cores) for i in range(cores)]
+    bounds = [b for b in bounds if b[1] > b[0]]
+    t0 = time.perf_counter()
+    with cf.ThreadPoolExecutor(len(bounds)) as ex:
+        res = list(ex.map(lambda b: oracle.compress_range(x, b[0], b[1]), bounds))
+    dt = time.perf_counter() - t0
+    nbytes = min(x.size, nchunks * S)
+    parity = None
+    if stream_bytes is not None:
+        sizes = np.concatenate([r[1] for r in res]).astype(np.int64)
+        payload = b"".join(r[0] for r in res)
+        Ctot = (x.size + S - 1) // S
+        gpu_sizes = np.frombuffer(stream_bytes, dtype="<u4", count=nchunks, offset=32).astype(np.int64)
+        start = 32 + 4 * Ctot
+        parity = bool(np.array_equal(sizes, gpu_sizes)
+                      and stream_bytes[start:start + len(payload)] == payload)
+    return {"value": nbytes / dt / 1e9, "unit": UNIT, "cores": len(bounds), "kind": "oracle",
+            "sample": f"first {nchunks} chunks ({nbytes} B) of the same input, {len(bounds)} threads "
+                      f"over contiguous chunk ranges, {dt:.2f} s wall",
+            "parity_with_gpu_stream": parity}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle (the only reference there is: the
+    paper ships no code) on the host cores, same metric/config/unit."""
+    if rank != 0:
+        return
+    import concurrent.futures as cf
+    import oracle
+    x = rank_input(args.config, 0, 1)
+    S = 4096
+    cores = max(1, min(len(os.sched_getaffinity(0)), 64))
+    C = (x.size + S - 1) // S
+    t0 = time.perf_counter()
+    oracle.compress_range(x, 0, min(C, 8))
+    per_chunk = (time.perf_counter() - t0) / min(C, 8)
+    # each step ~ (10 s / (steps + warmup)) of wall so the run stays within minutes
+    step_budget = max(0.5, 12.0 / (args.steps + args.warmup))
+    nchunks = int(min(C, max(cores, step_budget * cores / max(per_chunk, 1e-6))))
+    bounds = [(i * nchunks // cores, (i + 1) * nchunks // cores) for i in range(cores)]
+    bounds = [b for b in bounds if b[1] > b[0]]
+    times = []
+    out_bytes = 0
+    with cf.ThreadPoolExecutor(len(bounds)) as ex:
+        for it in range(args.warmup + args.steps):
+            t0 = time.perf_counter()
+            res = list(ex.map(lambda b: oracle.compress_range(x, b[0], b[1]), bounds))
+            dt = time.perf_counter() - t0
+            if it >= args.warmup:
+                times.append(dt)
+            out_bytes = sum(len(r[0]) for r in res) + 4 * nchunks + 32
+    nbytes = min(x.size, nchunks * S)
+    ms = 1000 * statistics.mean(times)
+    value = nbytes / (ms / 1000) / 1e9
+    sample = (f"first {nchunks} chunks ({nbytes} B) of {args.config} per step, {len(bounds)} threads "
+              f"over contiguous chunk ranges")
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": f"{args.config}: {CONFIG_TEXT[args.config]}", "bytes": int(x.size),
+                   "sample_bytes_per_step": int(nbytes), "chunk": 4096, "window": 128,
+                   "max_match": 128, "min_match": 3},
+        "ratio": out_bytes / nbytes,
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": len(bounds), "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "gpu_launches": 0,
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse_args()
+    rank, world, local = dist_env()
+    if world != args.gpus and world > 1:
+        print(f"warning: WORLD_SIZE={world} but --gpus {args.gpus}", file=sys.stderr)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_cluster_ozsoys11_b200 import culzss
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    x_np = rank_input(args.config, rank, world)
+    n = int(x_np.size)
+    x = torch.from_numpy(x_np).to(dev)
+    S = 4096
+    C = (n + S - 1) // S
+    out = torch.empty(culzss.max_compressed_size(n), dtype=torch.uint8, device=dev)
+    payload = out[32 + 4 * C:]
+    sizes = torch.empty(max(C, 1), dtype=torch.int32, device=dev)
+    totals = torch.zeros(world, dtype=torch.int64, device=dev)
+    mytotal = torch.zeros(1, dtype=torch.int64, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+    stream = torch.cuda.current_stream()
+    culzss.set_profiling(True)
+
+    def step():
+        if world == 1:
+            return culzss.compress_into(x, out), culzss.last_kernel_ms("call")
+        t = culzss.compress_chunks(x, payload, sizes)
+        ms_lib = culzss.last_kernel_ms("call")
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        mytotal.fill_(t)
+        dist.all_gather_into_tensor(totals, mytotal)
+        ev1.record(stream)
+        ev1.synchronize()
+        return t, ms_lib + ev0.elapsed_time(ev1)
+
+    for _ in range(args.warmup):
+        flush.fill_(1)
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = ClockSampler(local)
+    clocks.start()
+    launches0 = culzss.launch_count()
+    step_ms, chunk_ms, scan_ms, compact_ms = [], [], [], []
+    out_n = 0
+    for _ in range(args.steps):
+        flush.fill_(1)
+        torch.cuda.synchronize()
+        r, ms = step()
+        out_n = r
+        step_ms.append(ms)
+        chunk_ms.append(culzss.last_kernel_ms("chunk"))
+        scan_ms.append(culzss.last_kernel_ms("scan"))
+        compact_ms.append(culzss.last_kernel_ms("compact"))
+    torch.cuda.synchronize()
+    launches = culzss.launch_count() - launches0
+    clk = clocks.stop()
+    total_ms = sum(step_ms)
+    if world > 1:
+        t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+        dist.barrier()
+    ms_per_step = total_ms / args.steps
+    # global bytes: every rank holds n bytes (weak scaling)
+    n_total = n * world
+    value = n_total / (ms_per_step / 1000) / 1e9
+    if world == 1:
+        stream_len = out_n
+    else:
+        stream_len = 32 + 4 * C * world + int(totals.sum().item())
+    ratio = stream_len / n_total
+
+    # roofline of the dominant kernel (fused chunk kernel): algorithmic HBM
+    # bytes = read n + write the payload (sum of sizes) + 4 B size per chunk
+    hbm_peak, sm_max_mhz, peak_kind = load_peaks()
+    pay_bytes = (out_n - 32 - 4 * C) if world == 1 else int(totals[rank].item())
+    alg_bytes = n + pay_bytes + 4 * C
+    ck = statistics.mean(chunk_ms)
+    achieved = alg_bytes / (ck / 1000) / 1e9
+    # context: the survey's brute-force compare roofline:
+    # 125.98 byte-pair tests per input byte at 4 per 32-bit op, against
+    # 148 SM x 128 INT32 lanes/clk x sm_max clock
+    int_peak = 148 * 128 * sm_max_mhz * 1e6
+    t_cmp = 125.98 * n / 4 / int_peak * 1000
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": f"{args.config}: {CONFIG_TEXT[args.config]}", "bytes_per_rank": n,
+                   "chunk": 4096, "window": 128, "max_match": 128, "min_match": 3,
+                   "l2": "flushed (256 MiB write) between steps", "parallelism": f"dp{world} (chunk ranges)",
+                   "exchange": "NCCL all_gather of per-rank compressed totals" if world > 1 else "none"},
+        "ratio": ratio,
+        "kernels_ms": {"chunk": ck, "scan": statistics.mean(scan_ms), "compact": statistics.mean(compact_ms)},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+                     "frac": achieved / hbm_peak, "traffic": None, "peak_kind": peak_kind,
+                     "kernel": "chunk_kernel (fused a1-a4)", "algorithmic_bytes": alg_bytes,
+                     "alu_context": {"bruteforce_pair_tests_per_byte": 125.98, "int32_peak_tops": int_peak / 1e12,
+                                     "t_cmp_ms": t_cmp, "chunk_kernel_vs_t_cmp": t_cmp / ck}},
+        "clocks": clk,
+        "gpu_launches": launches,
+    }
+    # e2e through the public API with host buffers (pinned), N=1 only per rank
+    if not args.no_e2e:
+        hin = torch.from_numpy(x_np).pin_memory()
+        hout = torch.empty(culzss.max_compressed_size(n), dtype=torch.uint8).pin_memory()
+        times = []
+        on = 0
+        for it in range(args.warmup + max(3, args.steps // 2)):
+            ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            ev0.record(stream)
+            on = culzss.compress_host_ptr(hin.data_ptr(), n, hout.data_ptr(), hout.numel())
+            ev1.record(stream)
+            ev1.synchronize()
+            if it >= args.warmup:
+                times.append(ev0.elapsed_time(ev1))
+        e2e_ms = statistics.mean(times)
+        if world > 1:
+            t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_ms = float(t.item())
+        line["e2e"] = {"value": n_total / (e2e_ms / 1000) / 1e9, "unit": UNIT,
+                       "h2d_bytes_per_step": n, "d2h_bytes_per_step": int(on),
+                       "api": "culzss_compress_host (pinned host in/out)"}
+    if rank == 0 and not args.no_cpu_baseline:
+        sb = out[:out_n].cpu().numpy().tobytes() if world == 1 else None
+        line["cpu_baseline"] = cpu_baseline(x_np, sb)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()

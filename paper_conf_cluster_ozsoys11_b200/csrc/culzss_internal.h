@@ -9,30 +9,47 @@ namespace culzss {
 
 // Geometry of the fused chunk kernel.
 constexpr int kChunkMax = 4096;     // largest chunk the kernel stages (S <= 4096)
-constexpr int kSeg = 128;           // positions per lane in the parse (32 x 128 = 4096)
-constexpr int kHashBits = 10;       // 3-gram hash table: 1024 heads per chunk
-constexpr int kWarpsPerCta = 4;     // one warp per chunk
+constexpr int kSeg = 128;           // positions per lane segment (32 x 128 = 4096)
+constexpr int kHashBits = 8;        // per-lane 3-gram hash table: 256 heads
+constexpr int kWarpsPerCta = 3;     // one warp per chunk
 constexpr int kCtasPerSm = 3;
 
 struct Geometry {
     uint32_t S, W, F;               // chunk, window, max match (MIN is 3)
 };
 
-// Per-warp shared memory.  The output words alias link/head, which are dead
-// once the parse finishes.
+// Per-warp shared memory.  Per-position arrays use a SKEWED layout: 4 pad
+// bytes after every 128-position segment, so that the 32 lanes (one segment
+// each) scanning the same relative offset hit 32 different banks.  The pad
+// word of a segment duplicates the first word of the next one, so an
+// unaligned 4-byte load is two aligned word loads anywhere in the chunk.
+// During the chain build `tab` holds the per-lane hash heads; afterwards the
+// same bytes hold the walk stamps, per-walk exits and memoised tokens
+// (`ld`).  After the walks link/stamp/exits become per-lane bit staging and
+// `ld` the packed payload words.
+constexpr int kMaxWalks = 34;                        // speculative walk + <= 32 fix-up rounds
+constexpr int kSkewBytes = kChunkMax + 4 * (kChunkMax / kSeg);   // 4224
+constexpr int kStageWords = 69;                      // 128 tokens x 17 bits + 1; odd stride
 struct __align__(16) WarpSmem {
-    uint32_t cw[(kChunkMax + 16) / 4];                 // chunk bytes + zero pad
-    uint16_t ld[kChunkMax];                            // token at parse positions
+    uint32_t cw[(kSkewBytes + 16) / 4];              // chunk bytes (skewed) + zero tail
     union {
         struct {
-            uint8_t link[kChunkMax];                   // distance to previous same-hash position
-            uint16_t head[1 << kHashBits];             // latest position per hash
-        } s;
-        uint32_t ow[(kChunkMax + 2 * (1 << kHashBits)) / 4];   // packed payload words
-    } u;
+            uint8_t link[kSkewBytes];                // distance to previous same-hash position
+            union {
+                uint16_t tab[(1 << kHashBits) * 32]; // [hash][lane] -> position + 0x1000
+                struct {
+                    uint8_t stamp[kSkewBytes];       // walk index that started a token here
+                    uint16_t exits[32 * kMaxWalks];  // [lane][walk] -> exit position
+                    uint16_t ld[kChunkMax + 2 * (kChunkMax / kSeg)];  // memoised token (0 = not evaluated)
+                } w;
+            } u;
+        } a;
+        uint32_t stage[32 * kStageWords];            // per-lane bit staging (after walks)
+    } v;
 };
-static_assert(sizeof(WarpSmem) == 18448, "smem layout");
-static_assert((kChunkMax * 9 + 7) / 8 + 8 <= sizeof(WarpSmem::u), "payload fits alias");
+static_assert(sizeof(WarpSmem) <= 24848, "smem layout");
+static_assert(32 * kStageWords * 4 <= 2 * kSkewBytes + 32 * kMaxWalks * 2, "staging must not reach ld");
+static_assert((kChunkMax * 9 / 8 + 16) <= sizeof(WarpSmem::v.a.u.w.ld), "payload words fit in ld");
 
 __host__ __device__ inline uint64_t bucket_stride(uint32_t S) { return (((uint64_t)S * 9 + 7) / 8 + 15) / 16 * 16; }
 

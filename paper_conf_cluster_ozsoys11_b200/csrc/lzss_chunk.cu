@@ -13,26 +13,32 @@
 //   a4  bit-pack  flag 0 + byte | flag 1 + (D-1) + (L-3), MSB first, zero pad
 //                 (PAPER.md:1@4785, @23049-23282; readings R9-R11)
 //
-// B200 design, one warp per chunk, everything in shared memory:
-//   * Phase 1 builds exact 3-gram hash chains over the chunk, 32 positions per
-//     step: __match_any_sync groups equal hashes inside the step, a 1024-entry
-//     head table carries the latest position across steps.  link[p] = distance
-//     to the previous position with the same hash (0 = none within W).
-//     Every d with run_d(p) >= 3 shares p's 3-gram, hence its hash, so walking
-//     the chain while the distance stays <= W visits every candidate, nearest
-//     first -- the window-offset search of the paper without the brute force.
-//   * Phase 2 parses: lane l owns the 128-position segment [128l, 128l+128)
-//     and runs the greedy parse from its segment start speculatively,
-//     evaluating L/D only where its parse lands (the V1 "jump over" saving,
-//     PAPER.md:1@32329 §V).  Rounds of shuffles then hand each lane the true
-//     entry point (the previous lane's exit); a lane whose entry moved
-//     re-parses only until it meets its own earlier path, after which the
-//     greedy path is identical.  The result is the exact serial greedy parse.
-//   * Phase 3 bit-packs: per-lane bit counts, warp exclusive scan, each lane
-//     ORs its tokens into the payload words.
+// B200 design, one warp per chunk, everything in shared memory,
+// lane l owns the 128-position segment [128l, 128l + 128):
+//   * Chain build (a2, part 1).  Each lane inserts the W positions before its
+//     segment and then its own positions, in order, into its own 256-entry
+//     3-gram hash table, recording link[p] = distance to the previous
+//     position with the same hash (0 = none within W).  Every d with
+//     run_d(p) >= 3 shares p's 3-gram, hence its hash, so walking the chain
+//     while the distance stays <= W visits every candidate, nearest first --
+//     the paper's window-offset search without the brute force.  Per-lane
+//     tables make the build a straight-line loop (no intra-warp conflicts).
+//   * Lazy greedy walk (a2 part 2 + a3).  Each lane runs the greedy parse
+//     over its segment from the segment start, evaluating L/D only where the
+//     parse lands -- the V1 "jump over" saving (PAPER.md:1@32329 §V).  The
+//     walk is one flat state machine per lane (each iteration: one candidate
+//     word compare, or the start of a token), so lanes do not serialise on
+//     nested loops; runs of positions with no candidate are emitted as
+//     literals in one step from a 128-bit candidate mask.  Rounds of shuffles
+//     then hand each lane its true entry (the previous lane's exit); a lane
+//     whose entry moved re-walks only until it meets its earlier path, after
+//     which the greedy path is identical.  The result is exactly the serial
+//     greedy parse.
+//   * Bit-pack (a4): per-lane bit counts, warp exclusive scan, each lane ORs
+//     its tokens into the payload words.
 //
-// The match search compares 4 bytes per step (XOR of two 32-bit words, first
-// differing byte by __ffs), i.e. packed byte compares with early out.
+// The match extension compares 4 bytes per step (XOR of two 32-bit words,
+// first differing byte by __ffs): packed byte compares with early out.
 
 #include "culzss_internal.h"
 
@@ -40,104 +46,174 @@ namespace culzss {
 namespace {
 
 constexpr uint32_t kFull = 0xffffffffu;
-constexpr uint16_t kLiteral = 0xFFFF;
-constexpr uint16_t kNoPos = 0xFFFF;
+constexpr uint32_t kTabBias = 0x1000;   // table entry = position + bias; 0 = empty
+constexpr uint32_t kHashMul = 0x9E3779B1u << 8;
+// memoised token encoding in ld[]: 0 = not evaluated, 1 = literal,
+// 2 + (((D-1) << 8) | (L-3)) = match
+constexpr uint16_t kLit = 1;
+
+// skewed byte index of chunk position x (4 pad bytes per 128 positions)
+__device__ __forceinline__ int sk(int x) { return x + ((x >> 7) << 2); }
+// skewed u16 index of position x
+__device__ __forceinline__ int sk2(int x) { return x + ((x >> 7) << 1); }
 
 __device__ __forceinline__ uint32_t load4(const uint32_t *cw, int x) {
-    // bytes x..x+3 of the chunk (little endian), from two aligned words
-    uint32_t lo = cw[x >> 2], hi = cw[(x >> 2) + 1];
-    return __funnelshift_r(lo, hi, (x & 3) * 8);
+    // bytes x..x+3 of the chunk (little endian), from two aligned words; the
+    // pad word after each segment repeats the next segment's first word
+    const int a = sk(x);
+    const uint32_t lo = cw[a >> 2], hi = cw[(a >> 2) + 1];
+    return __funnelshift_r(lo, hi, (a & 3) * 8);
 }
 
 __device__ __forceinline__ uint32_t byte_at(const uint32_t *cw, int x) {
-    return reinterpret_cast<const uint8_t *>(cw)[x];
+    return reinterpret_cast<const uint8_t *>(cw)[sk(x)];
 }
 
-__device__ __forceinline__ uint32_t hash3(uint32_t key24) {
-    return (key24 * 0x9E3779B1u) >> (32 - kHashBits);
-}
+// byte offset (into the per-lane-interleaved table) of the 3-gram hash of a
+// little-endian word whose low 3 bytes are the 3-gram: hash h = top 8 bits of
+// (w << 8) * K (== w * (K << 8)); entry [h][lane] lives at byte 64 h + 2 lane
+__device__ __forceinline__ uint32_t hash_off(uint32_t w) { return ((w * kHashMul) >> 18) & 0x3FC0u; }
 
-// Longest common prefix of chunk[q..] and chunk[p..], capped at cap (>= 1).
-// Reads at most 3 bytes past p + cap (zero pad covers m + 16).
-__device__ __forceinline__ int lcp(const uint32_t *cw, int q, int p, int cap) {
-    int k = 0;
-    while (true) {
-        uint32_t x = load4(cw, q + k) ^ load4(cw, p + k);
-        if (x) {
-            k += (__ffs(x) - 1) >> 3;
-            break;
-        }
-        k += 4;
-        if (k >= cap) break;
+__device__ __forceinline__ int tok_len(uint32_t t) { return t == kLit ? 1 : ((t - 2) & 0xFF) + 3; }
+
+// first set bit at index >= off of the 128-bit mask {hi:lo}, 128 if none
+__device__ __forceinline__ int next_set(uint64_t lo, uint64_t hi, int off) {
+    if (off < 64) {
+        const uint64_t x = lo >> off;
+        if (x) return off + __ffsll(x) - 1;
+        return hi ? 63 + __ffsll(hi) : 128;
     }
-    return k < cap ? k : cap;
+    if (off >= 128) return 128;
+    const uint64_t y = hi >> (off - 64);
+    return y ? off + __ffsll(y) - 1 : 128;
+}
+__device__ __forceinline__ bool test128(uint64_t lo, uint64_t hi, int off) {
+    return ((off < 64 ? lo >> off : hi >> (off - 64)) & 1ull) != 0;
 }
 
-// Token at position p: ((D-1) << 8) | (L-3) for a match, kLiteral otherwise.
-__device__ __forceinline__ uint16_t eval_pos(const uint32_t *cw, const uint8_t *link, int p, int m,
-                                             int W, int F) {
-    int cap = min(F, m - p);
-    if (cap < 3) return kLiteral;
-    int d = link[p];
+// Token at one position by a plain chain walk (debug entry point only).
+__device__ uint32_t eval_pos(const uint32_t *cw, const uint8_t *link, int p, int m, int W, int F) {
+    const int cap = min(F, m - p);
+    if (cap < 3) return kLit;
+    int d = link[sk(p)];
     int bestL = 2, bestD = 0;
     while (d) {
-        int q = p - d;
-        // a candidate can only win if it also matches at offset bestL
-        if (bestL < 3 || byte_at(cw, q + bestL) == byte_at(cw, p + bestL)) {
-            int L = lcp(cw, q, p, cap);
-            if (L > bestL) {
-                bestL = L;
-                bestD = d;
-                if (L == cap) break;
+        const int q = p - d;
+        int k = 0;
+        while (true) {
+            const uint32_t x = load4(cw, q + k) ^ load4(cw, p + k);
+            if (x) {
+                k += (__ffs(x) - 1) >> 3;
+                break;
+            }
+            k += 4;
+            if (k >= cap) break;
+        }
+        const int L = min(k, cap);
+        if (L > bestL) {
+            bestL = L;
+            bestD = d;
+            if (L == cap) break;
+        }
+        const int l2 = link[sk(q)];
+        if (!l2 || d + l2 > W) break;
+        d += l2;
+    }
+    return bestD ? 2u + (((uint32_t)(bestD - 1) << 8) | (uint32_t)(bestL - 3)) : kLit;
+}
+
+__device__ __forceinline__ uint16_t enc_tok(int bestL, int bestD) {
+    return bestD ? (uint16_t)(2u + (((uint32_t)(bestD - 1) << 8) | (uint32_t)(bestL - 3))) : kLit;
+}
+
+// Speculative greedy walk over segment [s0, s1) from s0 as a branch-free
+// state machine: every iteration of every active lane does exactly one
+// 4-byte compare of its current candidate d at offset `off` and then updates
+// its state with selects:
+//   * a candidate first gets a reject test at offset bestL-3 (it can only
+//     win if bytes [0, bestL] match), then its LCP 4 bytes per iteration;
+//   * a finished candidate moves to the next one on the hash chain
+//     (d += link[p-d]) or finishes the token;
+//   * a finished token is memoised in ld[], its start stamped, and p jumps
+//     to the next candidate position (candidate-free positions are literals);
+//     the new token's first candidate is loaded in the same iteration.
+// Returns the exit (first position >= s1 the greedy path reaches).
+__device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link,
+                                         uint16_t *__restrict__ ld, uint8_t *__restrict__ stamp, int m, int W,
+                                         int F, int s0, int s1, uint64_t cm_lo, uint64_t cm_hi) {
+    int p = s0 < s1 ? min(s0 + next_set(cm_lo, cm_hi, 0), s1) : s0;
+    bool active = p < s1;
+    int d = 0, cap = 0;
+    if (active) {
+        d = link[sk(p)];
+        cap = min(F, m - p);
+        stamp[sk(p)] = 1;
+    }
+    int k = 0, bestL = 2, bestD = 0;
+    bool qr = false;
+#pragma unroll 1
+    while (__any_sync(kFull, active)) {
+        if (active) {
+            const int q = p - d;
+            const int off = qr ? bestL - 3 : k;
+            const uint32_t x = load4(cw, q + off) ^ load4(cw, p + off);
+            const int fb = x ? (__ffs(x) - 1) >> 3 : 4;
+            const bool cand_done = qr ? (x != 0) : (x != 0 || k + 4 >= cap);
+            const int L = min(k + fb, cap);
+            const bool upd = !qr && cand_done && L > bestL;
+            bestL = upd ? L : bestL;
+            bestD = upd ? d : bestD;
+            k = qr ? 0 : k + 4;
+            qr = qr && x != 0;
+            bool tok_done = false;
+            if (cand_done) {
+                const int l2 = bestL == cap ? 0 : link[sk(q)];
+                const int nd = d + l2;
+                tok_done = l2 == 0 || nd > W;
+                d = nd;
+                k = 0;
+                qr = bestL >= 3;
+            }
+            if (tok_done) {
+                ld[sk2(p)] = enc_tok(bestL, bestD);
+                p += bestD ? bestL : 1;
+                p = p < s1 ? min(s0 + next_set(cm_lo, cm_hi, p - s0), s1) : p;
+                active = p < s1;
+                if (active) {
+                    d = link[sk(p)];
+                    cap = min(F, m - p);
+                    stamp[sk(p)] = 1;
+                }
+                bestL = 2;
+                bestD = 0;
+                k = 0;
+                qr = false;
             }
         }
-        int l2 = link[q];
-        if (!l2) break;
-        d += l2;
-        if (d > W) break;
     }
-    return bestD ? (uint16_t)(((bestD - 1) << 8) | (bestL - 3)) : kLiteral;
+    return p;
 }
 
-__device__ __forceinline__ int tok_len(uint16_t t) { return t == kLiteral ? 1 : (t & 0xFF) + 3; }
-
-__device__ __forceinline__ bool mask_test(uint64_t lo, uint64_t hi, int off) {
-    return off < 64 ? (lo >> off) & 1ull : (hi >> (off - 64)) & 1ull;
-}
-__device__ __forceinline__ void mask_set(uint64_t &lo, uint64_t &hi, int off) {
-    if (off < 64) lo |= 1ull << off; else hi |= 1ull << (off - 64);
-}
-
-// Walk the greedy parse from `entry` inside segment [s0, s1) until the walk
-// leaves the segment or lands on a position of the current path (lo, hi).
-// On return (lo, hi) is the path from `entry` and exitp its exit.
-__device__ __forceinline__ void walk(const uint32_t *cw, const uint8_t *link, uint16_t *ld, int m,
-                                     int W, int F, int s0, int s1, int entry, uint64_t &lo,
-                                     uint64_t &hi, int &exitp) {
-    uint64_t nlo = 0, nhi = 0;
+// Re-walk from a corrected entry (fix-up rounds; short).  Candidate token
+// starts are stamped with `widx`; reaching a position stamped by an earlier
+// walk adopts that walk's exit (the greedy path from there is the same);
+// tokens memoised by earlier walks cost one lookup.
+__device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link,
+                        uint16_t *__restrict__ ld, uint8_t *__restrict__ stamp, const uint16_t *__restrict__ exits,
+                        int m, int W, int F, int s0, int s1, uint64_t cm_lo, uint64_t cm_hi, int entry, int widx) {
     int p = entry;
-    while (p < s1) {
-        int off = p - s0;
-        if (mask_test(lo, hi, off)) break;
-        uint16_t t = eval_pos(cw, link, p, m, W, F);
-        ld[p] = t;
-        mask_set(nlo, nhi, off);
-        p += tok_len(t);
-    }
-    if (p < s1) {  // merged with the old path at p: keep its positions >= p
-        int off = p - s0;
-        if (off < 64) {
-            lo &= ~0ull << off;
-        } else {
-            lo = 0;
-            hi &= ~0ull << (off - 64);
+    while (true) {
+        if (p < s1 && !test128(cm_lo, cm_hi, p - s0)) p = min(s0 + next_set(cm_lo, cm_hi, p - s0), s1);
+        if (p >= s1) return p;
+        const int st = stamp[sk(p)];
+        if (st) return exits[st];
+        stamp[sk(p)] = (uint8_t)widx;
+        uint32_t t = ld[sk2(p)];
+        if (!t) {
+            t = eval_pos(cw, link, p, m, W, F);
+            ld[sk2(p)] = (uint16_t)t;
         }
-        lo |= nlo;
-        hi |= nhi;
-    } else {
-        lo = nlo;
-        hi = nhi;
-        exitp = p;
+        p += tok_len(t);
     }
 }
 
@@ -157,150 +233,236 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     const int W = g.W, F = g.F;
     const uint8_t *src = in + start;
     uint8_t *cb = reinterpret_cast<uint8_t *>(sm.cw);
+    uint8_t *link = sm.v.a.link;
 
     // ---------------- a1: stage the chunk (16-byte coalesced loads) --------
+    {
+        uint4 *z4 = reinterpret_cast<uint4 *>(sm.cw);
+        const uint4 z = make_uint4(0, 0, 0, 0);
+        for (int i = lane; i < (int)(sizeof(sm.cw) / 16); i += 32) z4[i] = z;
+        uint4 *t4 = reinterpret_cast<uint4 *>(sm.v.a.u.tab);
+#pragma unroll 4
+        for (int i = lane; i < (int)(sizeof(sm.v.a.u.tab) / 16); i += 32) t4[i] = z;
+    }
+    __syncwarp();
     if ((reinterpret_cast<uintptr_t>(src) & 15) == 0) {
+        // a 16-byte group never straddles a 128-position segment
         const int nvec = m >> 4;
         const uint4 *s4 = reinterpret_cast<const uint4 *>(src);
-        uint4 *d4 = reinterpret_cast<uint4 *>(sm.cw);
-        for (int i = lane; i < nvec; i += 32) d4[i] = __ldcs(s4 + i);
-        for (int i = (nvec << 4) + lane; i < m; i += 32) cb[i] = src[i];
+        for (int i = lane; i < nvec; i += 32) {
+            const uint4 v = __ldcs(s4 + i);
+            uint32_t *d = sm.cw + (sk(i << 4) >> 2);
+            d[0] = v.x;
+            d[1] = v.y;
+            d[2] = v.z;
+            d[3] = v.w;
+        }
+        for (int i = (nvec << 4) + lane; i < m; i += 32) cb[sk(i)] = src[i];
     } else {
-        for (int i = lane; i < m; i += 32) cb[i] = src[i];
+        for (int i = lane; i < m; i += 32) cb[sk(i)] = src[i];
     }
-    if (lane < 16) cb[m + lane] = 0;  // zero pad: lcp may read 3 bytes past m
-    for (int i = lane; i < (1 << kHashBits) / 2; i += 32)
-        reinterpret_cast<uint32_t *>(sm.u.s.head)[i] = 0xFFFFFFFFu;
+    __syncwarp();
+    // pad word of segment `lane` = first word of the next segment (0 past the end)
+    sm.cw[33 * lane + 32] = lane < 31 ? sm.cw[33 * (lane + 1)] : 0u;
     __syncwarp();
 
-    // ---------------- a2 (part 1): 3-gram hash chains -----------------------
-    const uint32_t lt = (1u << lane) - 1u;
-    const uint32_t gt = ~lt & ~(1u << lane);
-    uint8_t *link = sm.u.s.link;
-    uint16_t *head = sm.u.s.head;
-    for (int base = 0; base < m; base += 32) {
-        const int p = base + lane;
-        const bool valid = p + 2 < m;
-        uint32_t h = 0x10000u + lane;  // unique dummy for lanes without a 3-gram
-        if (valid) h = hash3(load4(sm.cw, p) & 0xFFFFFFu);
-        const uint32_t grp = __match_any_sync(kFull, h);
-        if (p < m) {
-            uint32_t lk = 0;
-            if (valid) {
-                const uint32_t lower = grp & lt;
-                const int q = lower ? base + 31 - __clz(lower) : (int)head[h];
-                if (q != kNoPos && p - q <= W) lk = (uint32_t)(p - q);
-            }
-            link[p] = (uint8_t)lk;
+    // ---------------- a2 part 1: per-lane 3-gram hash chains ---------------
+    // Straight-line: every position is hashed and inserted; positions whose
+    // 3-gram would run past the chunk end (the last two) get link 0 after.
+    const int s0 = lane * kSeg;
+    const int s1 = min(s0 + kSeg, m);  // <= s0 for lanes past the chunk end
+    unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.v.a.u.tab) + 2 * lane;
+    uint32_t cmw0 = 0u, cmw1 = 0u, cmw2 = 0u, cmw3 = 0u;  // candidate mask words (link != 0)
+    if (s0 < m) {
+        // the W positions before the segment (pre-insert, no links)
+#pragma unroll 1
+        for (int q = max(0, s0 - W) & ~3; q < s0; q += 4) {
+            const uint32_t w0 = sm.cw[sk(q) >> 2], w1 = sm.cw[(sk(q) >> 2) + 1];
+#pragma unroll
+            for (int j = 0; j < 4; j++)
+                *reinterpret_cast<uint16_t *>(tabl + hash_off(__funnelshift_r(w0, w1, 8 * j))) =
+                    (uint16_t)(q + j + kTabBias);
         }
-        __syncwarp();
-        if (valid && !(grp & gt)) head[h] = (uint16_t)p;
-        __syncwarp();
+        // own segment: links, 32 positions per mask word
+#pragma unroll 1
+        for (int wi = 0; wi < 4; wi++) {
+            uint32_t mw = 0;
+            const int pb = s0 + 32 * wi;
+            if (pb < s1) {
+#pragma unroll
+                for (int i = 0; i < 8; i++) {
+                    const int p = pb + 4 * i;
+                    const uint32_t w0 = sm.cw[sk(p) >> 2], w1 = sm.cw[(sk(p) >> 2) + 1];
+                    uint32_t lw = 0;
+#pragma unroll
+                    for (int j = 0; j < 4; j++) {
+                        uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(__funnelshift_r(w0, w1, 8 * j)));
+                        const uint32_t dist = (uint32_t)(p + j + kTabBias) - *e;
+                        *e = (uint16_t)(p + j + kTabBias);
+                        lw |= (dist <= (uint32_t)W ? dist : 0u) << (8 * j);
+                    }
+                    *reinterpret_cast<uint32_t *>(link + sk(p)) = lw;
+                    // nonzero bytes -> 4 mask bits (multiply gathers bits 7,15,23,31)
+                    const uint32_t nz = (((lw & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | lw) & 0x80808080u;
+                    mw |= ((nz >> 7) * 0x10204080u >> 28) << (4 * i);
+                }
+            }
+            cmw0 = wi == 0 ? mw : cmw0;
+            cmw1 = wi == 1 ? mw : cmw1;
+            cmw2 = wi == 2 ? mw : cmw2;
+            cmw3 = wi == 3 ? mw : cmw3;
+        }
     }
+    uint64_t cm_lo = ((uint64_t)cmw1 << 32) | cmw0;
+    uint64_t cm_hi = ((uint64_t)cmw3 << 32) | cmw2;
+    // positions m-2 and m-1 have no 3-gram: never candidates
+#pragma unroll
+    for (int t = 1; t <= 2; t++) {
+        const int x = m - t;
+        if (x >= s0 && x < s1) {
+            const int off = x - s0;
+            link[sk(x)] = 0;
+            if (off < 64) cm_lo &= ~(1ull << off); else cm_hi &= ~(1ull << (off - 64));
+        }
+    }
+    __syncwarp();
 
     if (MODE == kModeDumpMatch) {
         // every position, for per-position parity (a2)
         uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
         for (int p = lane; p < m; p += 32) {
-            uint16_t t = eval_pos(sm.cw, link, p, m, W, F);
-            uint32_t L = t == kLiteral ? 0 : (t & 0xFF) + 3;
-            uint32_t D = t == kLiteral ? 0 : (t >> 8) + 1;
-            LD[2 * p] = (uint8_t)L;
-            LD[2 * p + 1] = (uint8_t)D;
+            const uint32_t t = eval_pos(sm.cw, link, p, m, W, F);
+            LD[2 * p] = (uint8_t)(t == kLit ? 0 : ((t - 2) & 0xFF) + 3);
+            LD[2 * p + 1] = (uint8_t)(t == kLit ? 0 : ((t - 2) >> 8) + 1);
         }
         return;
     }
 
-    // ---------------- a3: speculative segment-parallel greedy parse --------
-    const int s0 = lane * kSeg;
-    const int s1 = max(s0, min(s0 + kSeg, m));
-    uint64_t lo = 0, hi = 0;
-    int exitp = s0;
-    walk(sm.cw, link, sm.ld, m, W, F, s0, s1, s0, lo, hi, exitp);
+    // ---------------- a3: lazy greedy walk, speculative per segment --------
+    uint8_t *stamp = sm.v.a.u.w.stamp;
+    uint16_t *ld = sm.v.a.u.w.ld;
+    uint16_t *exits = sm.v.a.u.w.exits + lane * kMaxWalks;
+    {
+        // zero stamps and memoised tokens (their bytes held the hash tables)
+        uint32_t *z1 = reinterpret_cast<uint32_t *>(stamp);
+        for (int i = lane; i < kSkewBytes / 4; i += 32) z1[i] = 0u;
+        uint4 *l4 = reinterpret_cast<uint4 *>(ld);
+        const uint4 z = make_uint4(0, 0, 0, 0);
+        for (int i = lane; i < (int)(sizeof(sm.v.a.u.w.ld) / 16); i += 32) l4[i] = z;
+    }
+    __syncwarp();
+    int exitp = walk_spec(sm.cw, link, ld, stamp, m, W, F, s0, s1, cm_lo, cm_hi);
+    exits[1] = (uint16_t)exitp;
     int cur = s0;
+    int widx = 1;
+#pragma unroll 1
     while (true) {
         int entry = __shfl_up_sync(kFull, exitp, 1);
         if (lane == 0) entry = 0;
         const bool chg = entry != cur;
+        if (!__any_sync(kFull, chg)) break;
         if (chg) {
-            walk(sm.cw, link, sm.ld, m, W, F, s0, s1, entry, lo, hi, exitp);
+            widx++;
+            exitp = walk_fix(sm.cw, link, ld, stamp, exits, m, W, F, s0, s1, cm_lo, cm_hi, entry, widx);
+            exits[widx] = (uint16_t)exitp;
             cur = entry;
         }
-        if (!__any_sync(kFull, chg)) break;
     }
+    __syncwarp();
 
     if (MODE == kModeDumpTokens) {
         uint32_t *tok = reinterpret_cast<uint32_t *>(dbg) + start;
-        for (int p = s0; p < s1; p++) {
-            uint32_t v = 0;
-            if (mask_test(lo, hi, p - s0)) {
-                uint16_t t = sm.ld[p];
-                v = t == kLiteral ? 1u : ((uint32_t)((t & 0xFF) + 3) << 16) | ((t >> 8) + 1);
+        for (int p = s0; p < s1; p++) tok[p] = 0;
+        int p = cur;
+        while (p < s1) {
+            if (!test128(cm_lo, cm_hi, p - s0)) {
+                tok[p] = 1;
+                p++;
+            } else {
+                const uint32_t t = ld[sk2(p)];
+                tok[p] = t == kLit ? 1u : ((uint32_t)(((t - 2) & 0xFF) + 3) << 16) | (((t - 2) >> 8) + 1);
+                p += tok_len(t);
             }
-            tok[p] = v;
         }
         return;
     }
 
     // ---------------- a4: bit-pack ----------------------------------------
-    int nbits = 9 * __popcll(lo) + 9 * __popcll(hi);
+    // Each lane emits its path's tokens MSB-first into its own staging words
+    // starting at bit 0 (one token per loop iteration; a token is a literal,
+    // a pair of literals of a candidate-free run, or a match); after the warp
+    // scan of bit counts the staged words are shifted into place.
+    uint32_t *stage = sm.v.stage + lane * kStageWords;
+    int nbits = 0;
     {
-        uint64_t w = lo;
-        while (w) {
-            int b = __ffsll(w) - 1;
-            w &= w - 1;
-            if (sm.ld[s0 + b] != kLiteral) nbits += 8;
+        uint64_t acc = 0;
+        int nacc = 0, nw = 0;
+        int p = cur;
+        int run_end = p;  // end of the current candidate-free run
+#pragma unroll 1
+        while (p < s1) {
+            uint32_t val;
+            int nb, adv;
+            if (p < run_end || !test128(cm_lo, cm_hi, p - s0)) {
+                if (p >= run_end) run_end = min(s0 + next_set(cm_lo, cm_hi, p - s0), s1);
+                if (p + 2 <= run_end) {
+                    val = (byte_at(sm.cw, p) << 9) | byte_at(sm.cw, p + 1);
+                    nb = 18;
+                    adv = 2;
+                } else {
+                    val = byte_at(sm.cw, p);
+                    nb = 9;
+                    adv = 1;
+                }
+            } else {
+                const uint32_t t = ld[sk2(p)];
+                const bool lit = t == kLit;
+                val = lit ? byte_at(sm.cw, p) : 0x10000u | (t - 2);
+                nb = lit ? 9 : 17;
+                adv = lit ? 1 : ((t - 2) & 0xFF) + 3;
+            }
+            acc = (acc << nb) | val;
+            nacc += nb;
+            nbits += nb;
+            p += adv;
+            if (nacc >= 32) {
+                nacc -= 32;
+                stage[nw++] = (uint32_t)(acc >> nacc);
+            }
         }
-        w = hi;
-        while (w) {
-            int b = __ffsll(w) - 1;
-            w &= w - 1;
-            if (sm.ld[s0 + 64 + b] != kLiteral) nbits += 8;
-        }
+        if (nacc > 0) stage[nw] = (uint32_t)(acc << (32 - nacc));
     }
     int incl = nbits;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-        int y = __shfl_up_sync(kFull, incl, o);
+        const int y = __shfl_up_sync(kFull, incl, o);
         if (lane >= o) incl += y;
     }
     const int excl = incl - nbits;
     const int total = __shfl_sync(kFull, incl, 31);
     const int nwords = (total + 31) >> 5;
-    uint32_t *ow = sm.u.ow;
-    __syncwarp();  // link/head are dead from here on
+    uint32_t *ow = reinterpret_cast<uint32_t *>(ld);  // ld is dead: payload words
+    __syncwarp();
     for (int i = lane; i < nwords + 1; i += 32) ow[i] = 0;
     __syncwarp();
     {
-        uint64_t acc = 0;
-        int nacc = excl & 31;
-        int wi = excl >> 5;
+        // shift the lane's staged words to bit offset excl; output words shared
+        // with the neighbouring lanes (first, last, spill) are OR-ed atomically
+        const int sh = excl & 31;
+        const int base = excl >> 5;
+        const int nsw = (nbits + 31) >> 5;
+        uint32_t prev = 0;
 #pragma unroll 1
-        for (int half = 0; half < 2; half++) {
-            uint64_t w = half ? hi : lo;
-            while (w) {
-                const int b = __ffsll(w) - 1;
-                w &= w - 1;
-                const int p = s0 + half * 64 + b;
-                const uint16_t t = sm.ld[p];
-                uint32_t val;
-                int nb;
-                if (t == kLiteral) {
-                    val = cb[p];
-                    nb = 9;
-                } else {
-                    val = 0x10000u | t;
-                    nb = 17;
-                }
-                acc = (acc << nb) | val;
-                nacc += nb;
-                if (nacc >= 32) {
-                    nacc -= 32;
-                    atomicOr(&ow[wi++], (uint32_t)(acc >> nacc));
-                }
-            }
+        for (int i = 0; i < nsw; i++) {
+            const uint32_t v = stage[i];
+            const uint32_t o = sh ? (prev << (32 - sh)) | (v >> sh) : v;
+            if (i == 0 || i == nsw - 1) atomicOr(&ow[base + i], o); else ow[base + i] = o;
+            prev = v;
         }
-        if (nacc > 0) atomicOr(&ow[wi], (uint32_t)(acc << (32 - nacc)));
+        if (sh && nsw) {
+            const uint32_t o = prev << (32 - sh);
+            if (o) atomicOr(&ow[base + nsw], o);
+        }
     }
     __syncwarp();
 
