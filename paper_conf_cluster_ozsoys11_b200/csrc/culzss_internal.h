@@ -2,6 +2,7 @@
 // Not part of the ABI (the ABI is include/culzss.h).  Shares nothing with
 // oracle/ (independence rule).
 #pragma once
+#include <cstddef>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -24,32 +25,32 @@ struct Geometry {
 // word of a segment duplicates the first word of the next one, so an
 // unaligned 4-byte load is two aligned word loads anywhere in the chunk.
 // During the chain build `tab` holds the per-lane hash heads; afterwards the
-// same bytes hold the walk stamps, per-walk exits and memoised tokens
-// (`ld`).  After the walks link/stamp/exits become per-lane bit staging and
-// `ld` the packed payload words.
-constexpr int kMaxWalks = 34;                        // speculative walk + <= 32 fix-up rounds
+// same bytes hold nc[] (distance to the next candidate position) and the
+// memoised tokens (`ld`).  After the walks link/nc become per-lane bit
+// staging and `ld` the packed payload words.
 constexpr int kSkewBytes = kChunkMax + 4 * (kChunkMax / kSeg);   // 4224
-constexpr int kStageWords = 69;                      // 128 tokens x 17 bits + 1; odd stride
+// per-lane bit staging: a segment emits at most 9 bits per position (a 17-bit
+// match covers >= 3 positions) + one 17-bit token crossing its end: 37 words
+constexpr int kStageWords = 37;                      // odd stride: conflict-free
+constexpr int kStagePad = 32 * kStageWords * 4 - kSkewBytes;      // 512
 struct __align__(16) WarpSmem {
     uint32_t cw[(kSkewBytes + 16) / 4];              // chunk bytes (skewed) + zero tail
-    union {
-        struct {
-            uint8_t link[kSkewBytes];                // distance to previous same-hash position
-            union {
-                uint16_t tab[(1 << kHashBits) * 32]; // [hash][lane] -> position + 0x1000
-                struct {
-                    uint8_t stamp[kSkewBytes];       // walk index that started a token here
-                    uint16_t exits[32 * kMaxWalks];  // [lane][walk] -> exit position
-                    uint16_t ld[kChunkMax + 2 * (kChunkMax / kSeg)];  // memoised token (0 = not evaluated)
-                } w;
-            } u;
-        } a;
-        uint32_t stage[32 * kStageWords];            // per-lane bit staging (after walks)
-    } v;
+    struct {
+        uint8_t link[kSkewBytes];                    // distance to previous same-hash position
+        union {
+            uint16_t tab[(1 << kHashBits) * 32];     // [hash][lane] -> position + 0x1000
+            struct {
+                uint8_t pad[kStagePad];              // staging = link + pad (after the walks)
+                uint8_t nc[kSkewBytes];              // distance to next candidate position (<= s1)
+                uint16_t ld[kChunkMax + 2 * (kChunkMax / kSeg)];  // memoised token (0 = not evaluated)
+            } w;
+        } u;
+    } a;
 };
 static_assert(sizeof(WarpSmem) <= 24848, "smem layout");
-static_assert(32 * kStageWords * 4 <= 2 * kSkewBytes + 32 * kMaxWalks * 2, "staging must not reach ld");
-static_assert((kChunkMax * 9 / 8 + 16) <= sizeof(WarpSmem::v.a.u.w.ld), "payload words fit in ld");
+static_assert(offsetof(WarpSmem, a.u.w.nc) - offsetof(WarpSmem, a.link) >= 32 * kStageWords * 4,
+              "staging (over link + pad) must not reach nc");
+static_assert((kChunkMax * 9 / 8 + 16) <= sizeof(WarpSmem::a.u.w.ld), "payload words fit in ld");
 
 __host__ __device__ inline uint64_t bucket_stride(uint32_t S) { return (((uint64_t)S * 9 + 7) / 8 + 15) / 16 * 16; }
 

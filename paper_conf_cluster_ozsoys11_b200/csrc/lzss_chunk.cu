@@ -53,7 +53,7 @@ constexpr uint32_t kHashMul = 0x9E3779B1u << 8;
 constexpr uint16_t kLit = 1;
 
 // skewed byte index of chunk position x (4 pad bytes per 128 positions)
-__device__ __forceinline__ int sk(int x) { return x + ((x >> 7) << 2); }
+__device__ __forceinline__ int sk(int x) { return (int)((unsigned)x + (((unsigned)x >> 7) << 2)); }
 // skewed u16 index of position x
 __device__ __forceinline__ int sk2(int x) { return x + ((x >> 7) << 1); }
 
@@ -76,17 +76,6 @@ __device__ __forceinline__ uint32_t hash_off(uint32_t w) { return ((w * kHashMul
 
 __device__ __forceinline__ int tok_len(uint32_t t) { return t == kLit ? 1 : ((t - 2) & 0xFF) + 3; }
 
-// first set bit at index >= off of the 128-bit mask {hi:lo}, 128 if none
-__device__ __forceinline__ int next_set(uint64_t lo, uint64_t hi, int off) {
-    if (off < 64) {
-        const uint64_t x = lo >> off;
-        if (x) return off + __ffsll(x) - 1;
-        return hi ? 63 + __ffsll(hi) : 128;
-    }
-    if (off >= 128) return 128;
-    const uint64_t y = hi >> (off - 64);
-    return y ? off + __ffsll(y) - 1 : 128;
-}
 __device__ __forceinline__ bool test128(uint64_t lo, uint64_t hi, int off) {
     return ((off < 64 ? lo >> off : hi >> (off - 64)) & 1ull) != 0;
 }
@@ -126,6 +115,12 @@ __device__ __forceinline__ uint16_t enc_tok(int bestL, int bestD) {
     return bestD ? (uint16_t)(2u + (((uint32_t)(bestD - 1) << 8) | (uint32_t)(bestL - 3))) : kLit;
 }
 
+__device__ __forceinline__ void mark128(uint64_t &lo, uint64_t &hi, int off) {
+    const uint64_t bit = 1ull << (off & 63);
+    lo |= off < 64 ? bit : 0ull;
+    hi |= off < 64 ? 0ull : bit;
+}
+
 // Speculative greedy walk over segment [s0, s1) from s0 as a branch-free
 // state machine: every iteration of every active lane does exactly one
 // 4-byte compare of its current candidate d at offset `off` and then updates
@@ -134,20 +129,20 @@ __device__ __forceinline__ uint16_t enc_tok(int bestL, int bestD) {
 //     win if bytes [0, bestL] match), then its LCP 4 bytes per iteration;
 //   * a finished candidate moves to the next one on the hash chain
 //     (d += link[p-d]) or finishes the token;
-//   * a finished token is memoised in ld[], its start stamped, and p jumps
-//     to the next candidate position (candidate-free positions are literals);
-//     the new token's first candidate is loaded in the same iteration.
+//   * a finished token is memoised in ld[], its start marked in the lane's
+//     path mask, and p jumps over candidate-free positions (literals) with
+//     nc[]; the new token's first candidate is loaded in the same iteration.
 // Returns the exit (first position >= s1 the greedy path reaches).
 __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link,
-                                         uint16_t *__restrict__ ld, uint8_t *__restrict__ stamp, int m, int W,
-                                         int F, int s0, int s1, uint64_t cm_lo, uint64_t cm_hi) {
-    int p = s0 < s1 ? min(s0 + next_set(cm_lo, cm_hi, 0), s1) : s0;
+                                         const uint8_t *__restrict__ nc, uint16_t *__restrict__ ld, int m,
+                                         int W, int F, int s0, int s1, uint64_t &plo, uint64_t &phi) {
+    int p = s0 < s1 ? s0 + nc[sk(s0)] : s0;
     bool active = p < s1;
     int d = 0, cap = 0;
     if (active) {
         d = link[sk(p)];
         cap = min(F, m - p);
-        stamp[sk(p)] = 1;
+        mark128(plo, phi, p - s0);
     }
     int k = 0, bestL = 2, bestD = 0;
     bool qr = false;
@@ -177,12 +172,12 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const 
             if (tok_done) {
                 ld[sk2(p)] = enc_tok(bestL, bestD);
                 p += bestD ? bestL : 1;
-                p = p < s1 ? min(s0 + next_set(cm_lo, cm_hi, p - s0), s1) : p;
+                if (p < s1) p += nc[sk(p)];
                 active = p < s1;
                 if (active) {
                     d = link[sk(p)];
                     cap = min(F, m - p);
-                    stamp[sk(p)] = 1;
+                    mark128(plo, phi, p - s0);
                 }
                 bestL = 2;
                 bestD = 0;
@@ -194,20 +189,35 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const 
     return p;
 }
 
-// Re-walk from a corrected entry (fix-up rounds; short).  Candidate token
-// starts are stamped with `widx`; reaching a position stamped by an earlier
-// walk adopts that walk's exit (the greedy path from there is the same);
-// tokens memoised by earlier walks cost one lookup.
+// Re-walk from a corrected entry (fix-up rounds; short).  Reaching a token
+// start of the lane's current path (plo, phi) adopts that path's exit: the
+// greedy path from there is the same.  Tokens memoised by earlier walks cost
+// one lookup.  On return (plo, phi) is the new path, the result its exit.
 __device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link,
-                        uint16_t *__restrict__ ld, uint8_t *__restrict__ stamp, const uint16_t *__restrict__ exits,
-                        int m, int W, int F, int s0, int s1, uint64_t cm_lo, uint64_t cm_hi, int entry, int widx) {
+                        const uint8_t *__restrict__ nc, uint16_t *__restrict__ ld, int m, int W, int F, int s0,
+                        int s1, int entry, int old_exit, uint64_t &plo, uint64_t &phi) {
+    uint64_t nlo = 0, nhi = 0;
     int p = entry;
     while (true) {
-        if (p < s1 && !test128(cm_lo, cm_hi, p - s0)) p = min(s0 + next_set(cm_lo, cm_hi, p - s0), s1);
-        if (p >= s1) return p;
-        const int st = stamp[sk(p)];
-        if (st) return exits[st];
-        stamp[sk(p)] = (uint8_t)widx;
+        if (p < s1) p += nc[sk(p)];
+        if (p >= s1) {
+            plo = nlo;
+            phi = nhi;
+            return p;
+        }
+        const int off = p - s0;
+        if (test128(plo, phi, off)) {  // merged: keep the old path from p on
+            if (off < 64) {
+                plo &= ~0ull << off;
+            } else {
+                plo = 0;
+                phi &= ~0ull << (off - 64);
+            }
+            plo |= nlo;
+            phi |= nhi;
+            return old_exit;
+        }
+        mark128(nlo, nhi, off);
         uint32_t t = ld[sk2(p)];
         if (!t) {
             t = eval_pos(cw, link, p, m, W, F);
@@ -233,16 +243,16 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     const int W = g.W, F = g.F;
     const uint8_t *src = in + start;
     uint8_t *cb = reinterpret_cast<uint8_t *>(sm.cw);
-    uint8_t *link = sm.v.a.link;
+    uint8_t *link = sm.a.link;
 
     // ---------------- a1: stage the chunk (16-byte coalesced loads) --------
     {
         uint4 *z4 = reinterpret_cast<uint4 *>(sm.cw);
         const uint4 z = make_uint4(0, 0, 0, 0);
         for (int i = lane; i < (int)(sizeof(sm.cw) / 16); i += 32) z4[i] = z;
-        uint4 *t4 = reinterpret_cast<uint4 *>(sm.v.a.u.tab);
+        uint4 *t4 = reinterpret_cast<uint4 *>(sm.a.u.tab);
 #pragma unroll 4
-        for (int i = lane; i < (int)(sizeof(sm.v.a.u.tab) / 16); i += 32) t4[i] = z;
+        for (int i = lane; i < (int)(sizeof(sm.a.u.tab) / 16); i += 32) t4[i] = z;
     }
     __syncwarp();
     if ((reinterpret_cast<uintptr_t>(src) & 15) == 0) {
@@ -271,8 +281,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     // 3-gram would run past the chunk end (the last two) get link 0 after.
     const int s0 = lane * kSeg;
     const int s1 = min(s0 + kSeg, m);  // <= s0 for lanes past the chunk end
-    unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.v.a.u.tab) + 2 * lane;
-    uint32_t cmw0 = 0u, cmw1 = 0u, cmw2 = 0u, cmw3 = 0u;  // candidate mask words (link != 0)
+    unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + 2 * lane;
     if (s0 < m) {
         // the W positions before the segment (pre-insert, no links)
 #pragma unroll 1
@@ -283,10 +292,9 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                 *reinterpret_cast<uint16_t *>(tabl + hash_off(__funnelshift_r(w0, w1, 8 * j))) =
                     (uint16_t)(q + j + kTabBias);
         }
-        // own segment: links, 32 positions per mask word
+        // own segment: links
 #pragma unroll 1
         for (int wi = 0; wi < 4; wi++) {
-            uint32_t mw = 0;
             const int pb = s0 + 32 * wi;
             if (pb < s1) {
 #pragma unroll
@@ -302,28 +310,15 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                         lw |= (dist <= (uint32_t)W ? dist : 0u) << (8 * j);
                     }
                     *reinterpret_cast<uint32_t *>(link + sk(p)) = lw;
-                    // nonzero bytes -> 4 mask bits (multiply gathers bits 7,15,23,31)
-                    const uint32_t nz = (((lw & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | lw) & 0x80808080u;
-                    mw |= ((nz >> 7) * 0x10204080u >> 28) << (4 * i);
                 }
             }
-            cmw0 = wi == 0 ? mw : cmw0;
-            cmw1 = wi == 1 ? mw : cmw1;
-            cmw2 = wi == 2 ? mw : cmw2;
-            cmw3 = wi == 3 ? mw : cmw3;
         }
     }
-    uint64_t cm_lo = ((uint64_t)cmw1 << 32) | cmw0;
-    uint64_t cm_hi = ((uint64_t)cmw3 << 32) | cmw2;
     // positions m-2 and m-1 have no 3-gram: never candidates
 #pragma unroll
     for (int t = 1; t <= 2; t++) {
         const int x = m - t;
-        if (x >= s0 && x < s1) {
-            const int off = x - s0;
-            link[sk(x)] = 0;
-            if (off < 64) cm_lo &= ~(1ull << off); else cm_hi &= ~(1ull << (off - 64));
-        }
+        if (x >= s0 && x < s1) link[sk(x)] = 0;
     }
     __syncwarp();
 
@@ -339,22 +334,35 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     }
 
     // ---------------- a3: lazy greedy walk, speculative per segment --------
-    uint8_t *stamp = sm.v.a.u.w.stamp;
-    uint16_t *ld = sm.v.a.u.w.ld;
-    uint16_t *exits = sm.v.a.u.w.exits + lane * kMaxWalks;
+    uint8_t *nc = sm.a.u.w.nc;
+    uint16_t *ld = sm.a.u.w.ld;
     {
-        // zero stamps and memoised tokens (their bytes held the hash tables)
-        uint32_t *z1 = reinterpret_cast<uint32_t *>(stamp);
-        for (int i = lane; i < kSkewBytes / 4; i += 32) z1[i] = 0u;
+        // zero the memoised tokens (their bytes held the hash tables)
         uint4 *l4 = reinterpret_cast<uint4 *>(ld);
         const uint4 z = make_uint4(0, 0, 0, 0);
-        for (int i = lane; i < (int)(sizeof(sm.v.a.u.w.ld) / 16); i += 32) l4[i] = z;
+        for (int i = lane; i < (int)(sizeof(sm.a.u.w.ld) / 16); i += 32) l4[i] = z;
+    }
+    if (s0 < s1) {
+        // nc[p] = distance from p to the next candidate position (or to s1),
+        // one backward pass over the lane's link words
+        int nxt = s1;  // next candidate position after the current word
+#pragma unroll 1
+        for (int w = ((s1 - 1 - s0) >> 2); w >= 0; w--) {
+            const int p = s0 + 4 * w;
+            const uint32_t lw = *reinterpret_cast<const uint32_t *>(link + sk(p));
+            uint32_t out = 0;
+#pragma unroll
+            for (int j = 3; j >= 0; j--) {
+                nxt = (((lw >> (8 * j)) & 0xFFu) && p + j < s1) ? p + j : nxt;
+                out |= (uint32_t)(nxt - (p + j)) << (8 * j);
+            }
+            *reinterpret_cast<uint32_t *>(nc + sk(p)) = out;
+        }
     }
     __syncwarp();
-    int exitp = walk_spec(sm.cw, link, ld, stamp, m, W, F, s0, s1, cm_lo, cm_hi);
-    exits[1] = (uint16_t)exitp;
+    uint64_t plo = 0, phi = 0;  // token starts (candidate positions) of the current path
+    int exitp = walk_spec(sm.cw, link, nc, ld, m, W, F, s0, s1, plo, phi);
     int cur = s0;
-    int widx = 1;
 #pragma unroll 1
     while (true) {
         int entry = __shfl_up_sync(kFull, exitp, 1);
@@ -362,9 +370,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         const bool chg = entry != cur;
         if (!__any_sync(kFull, chg)) break;
         if (chg) {
-            widx++;
-            exitp = walk_fix(sm.cw, link, ld, stamp, exits, m, W, F, s0, s1, cm_lo, cm_hi, entry, widx);
-            exits[widx] = (uint16_t)exitp;
+            exitp = walk_fix(sm.cw, link, nc, ld, m, W, F, s0, s1, entry, exitp, plo, phi);
             cur = entry;
         }
     }
@@ -375,7 +381,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         for (int p = s0; p < s1; p++) tok[p] = 0;
         int p = cur;
         while (p < s1) {
-            if (!test128(cm_lo, cm_hi, p - s0)) {
+            if (nc[sk(p)]) {
                 tok[p] = 1;
                 p++;
             } else {
@@ -392,20 +398,19 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     // starting at bit 0 (one token per loop iteration; a token is a literal,
     // a pair of literals of a candidate-free run, or a match); after the warp
     // scan of bit counts the staged words are shifted into place.
-    uint32_t *stage = sm.v.stage + lane * kStageWords;
+    uint32_t *stage = reinterpret_cast<uint32_t *>(sm.a.link) + lane * kStageWords;  // link is dead
     int nbits = 0;
     {
         uint64_t acc = 0;
         int nacc = 0, nw = 0;
         int p = cur;
-        int run_end = p;  // end of the current candidate-free run
 #pragma unroll 1
         while (p < s1) {
             uint32_t val;
             int nb, adv;
-            if (p < run_end || !test128(cm_lo, cm_hi, p - s0)) {
-                if (p >= run_end) run_end = min(s0 + next_set(cm_lo, cm_hi, p - s0), s1);
-                if (p + 2 <= run_end) {
+            const int run = nc[sk(p)];  // candidate-free positions from p: literals
+            if (run) {
+                if (run >= 2) {
                     val = (byte_at(sm.cw, p) << 9) | byte_at(sm.cw, p + 1);
                     nb = 18;
                     adv = 2;
