@@ -11,7 +11,8 @@ namespace culzss {
 // Geometry of the fused chunk kernel.
 constexpr int kChunkMax = 4096;     // largest chunk the kernel stages (S <= 4096)
 constexpr int kSeg = 128;           // positions per lane segment (32 x 128 = 4096)
-constexpr int kHashBits = 8;        // per-lane 3-gram hash table: 256 heads
+constexpr int kHashBits = 8;        // per-lane 3-gram hash table, W > 128: 256 u16 heads
+constexpr int kHashBitsSmallW = 9;  // W <= 128: 512 u8 heads (relative positions)
 constexpr int kWarpsPerCta = 3;     // one warp per chunk
 constexpr int kCtasPerSm = 3;
 
@@ -38,7 +39,8 @@ struct __align__(16) WarpSmem {
     struct {
         uint8_t link[kSkewBytes];                    // distance to previous same-hash position
         union {
-            uint16_t tab[(1 << kHashBits) * 32];     // [hash][lane] -> position + 0x1000
+            uint16_t tab[(1 << kHashBits) * 32];     // [hash][lane]: u16 position + 0x1000 (W > 128)
+                                                     // or u8 position mod 256, 512 buckets (W <= 128)
             struct {
                 uint8_t pad[kStagePad];              // staging = link + pad (after the walks)
                 uint8_t nc[kSkewBytes];              // distance to next candidate position (<= s1)

@@ -73,6 +73,8 @@ __device__ __forceinline__ uint32_t byte_at(const uint32_t *cw, int x) {
 // little-endian word whose low 3 bytes are the 3-gram: hash h = top 8 bits of
 // (w << 8) * K (== w * (K << 8)); entry [h][lane] lives at byte 64 h + 2 lane
 __device__ __forceinline__ uint32_t hash_off(uint32_t w) { return ((w * kHashMul) >> 18) & 0x3FC0u; }
+// W <= 128 variant: 9-bit hash, u8 entries [h][lane] at byte 32 h + lane
+__device__ __forceinline__ uint32_t hash_off9(uint32_t w) { return ((w * kHashMul) >> 18) & 0x3FE0u; }
 
 __device__ __forceinline__ int tok_len(uint32_t t) { return t == kLit ? 1 : ((t - 2) & 0xFF) + 3; }
 
@@ -151,6 +153,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const 
         if (active) {
             const int q = p - d;
             const int off = qr ? bestL - 3 : k;
+            const int lq = link[sk(q)];  // next chain member, loaded with the compare words
             const uint32_t x = load4(cw, q + off) ^ load4(cw, p + off);
             const int fb = x ? (__ffs(x) - 1) >> 3 : 4;
             const bool cand_done = qr ? (x != 0) : (x != 0 || k + 4 >= cap);
@@ -162,7 +165,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const 
             qr = qr && x != 0;
             bool tok_done = false;
             if (cand_done) {
-                const int l2 = bestL == cap ? 0 : link[sk(q)];
+                const int l2 = bestL == cap ? 0 : lq;
                 const int nd = d + l2;
                 tok_done = l2 == 0 || nd > W;
                 d = nd;
@@ -227,7 +230,7 @@ __device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restri
     }
 }
 
-template <int MODE>
+template <int MODE, bool SMALLW>
 __global__ void __launch_bounds__(kWarpsPerCta * 32, kCtasPerSm)
 chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__restrict__ bucket,
              uint32_t *__restrict__ sizes, void *__restrict__ dbg) {
@@ -251,8 +254,11 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         const uint4 z = make_uint4(0, 0, 0, 0);
         for (int i = lane; i < (int)(sizeof(sm.cw) / 16); i += 32) z4[i] = z;
         uint4 *t4 = reinterpret_cast<uint4 *>(sm.a.u.tab);
+        // u8 tables: empty = (s0 - 129) mod 256 = 0x7F (even lanes) / 0xFF (odd)
+        const uint32_t e = SMALLW ? 0xFF7FFF7Fu : 0u;
+        const uint4 te = make_uint4(e, e, e, e);
 #pragma unroll 4
-        for (int i = lane; i < (int)(sizeof(sm.a.u.tab) / 16); i += 32) t4[i] = z;
+        for (int i = lane; i < (int)(sizeof(sm.a.u.tab) / 16); i += 32) t4[i] = te;
     }
     __syncwarp();
     if ((reinterpret_cast<uintptr_t>(src) & 15) == 0) {
@@ -281,16 +287,20 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     // 3-gram would run past the chunk end (the last two) get link 0 after.
     const int s0 = lane * kSeg;
     const int s1 = min(s0 + kSeg, m);  // <= s0 for lanes past the chunk end
-    unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + 2 * lane;
+    unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + (SMALLW ? lane : 2 * lane);
     if (s0 < m) {
         // the W positions before the segment (pre-insert, no links)
 #pragma unroll 1
         for (int q = max(0, s0 - W) & ~3; q < s0; q += 4) {
             const uint32_t w0 = sm.cw[sk(q) >> 2], w1 = sm.cw[(sk(q) >> 2) + 1];
 #pragma unroll
-            for (int j = 0; j < 4; j++)
-                *reinterpret_cast<uint16_t *>(tabl + hash_off(__funnelshift_r(w0, w1, 8 * j))) =
-                    (uint16_t)(q + j + kTabBias);
+            for (int j = 0; j < 4; j++) {
+                const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
+                if (SMALLW)
+                    tabl[hash_off9(key)] = (uint8_t)(q + j);
+                else
+                    *reinterpret_cast<uint16_t *>(tabl + hash_off(key)) = (uint16_t)(q + j + kTabBias);
+            }
         }
         // own segment: links
 #pragma unroll 1
@@ -304,9 +314,19 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                     uint32_t lw = 0;
 #pragma unroll
                     for (int j = 0; j < 4; j++) {
-                        uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(__funnelshift_r(w0, w1, 8 * j)));
-                        const uint32_t dist = (uint32_t)(p + j + kTabBias) - *e;
-                        *e = (uint16_t)(p + j + kTabBias);
+                        const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
+                        uint32_t dist;
+                        if (SMALLW) {
+                            // entries hold position mod 256: every live entry is
+                            // within 256 of p, the empty value maps to 0 or > 128
+                            uint8_t *e = tabl + hash_off9(key);
+                            dist = (uint32_t)(p + j - *e) & 0xFFu;
+                            *e = (uint8_t)(p + j);
+                        } else {
+                            uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(key));
+                            dist = (uint32_t)(p + j + kTabBias) - *e;
+                            *e = (uint16_t)(p + j + kTabBias);
+                        }
                         lw |= (dist <= (uint32_t)W ? dist : 0u) << (8 * j);
                     }
                     *reinterpret_cast<uint32_t *>(link + sk(p)) = lw;
@@ -410,15 +430,12 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
             int nb, adv;
             const int run = nc[sk(p)];  // candidate-free positions from p: literals
             if (run) {
-                if (run >= 2) {
-                    val = (byte_at(sm.cw, p) << 9) | byte_at(sm.cw, p + 1);
-                    nb = 18;
-                    adv = 2;
-                } else {
-                    val = byte_at(sm.cw, p);
-                    nb = 9;
-                    adv = 1;
-                }
+                // up to 3 literals (27 bits) per step from one 4-byte load
+                const uint32_t w = load4(sm.cw, p);
+                const uint32_t t3 = ((w & 0xFFu) << 18) | (((w >> 8) & 0xFFu) << 9) | ((w >> 16) & 0xFFu);
+                adv = min(run, 3);
+                nb = 9 * adv;
+                val = t3 >> (27 - nb);
             } else {
                 const uint32_t t = ld[sk2(p)];
                 const bool lit = t == kLit;
@@ -487,7 +504,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     if (lane == 0) sizes[c] = (uint32_t)nbytes;
 }
 
-template <int MODE>
+template <int MODE, bool SMALLW>
 cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *bucket,
                         uint32_t *sizes, void *dbg, cudaStream_t st) {
     const uint64_t C = (n + g.S - 1) / g.S;
@@ -495,16 +512,22 @@ cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *buck
     const size_t smem = sizeof(WarpSmem) * kWarpsPerCta;
     static bool attr_set = false;  // benign race: idempotent
     if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(chunk_kernel<MODE>,
+        cudaError_t e = cudaFuncSetAttribute(chunk_kernel<MODE, SMALLW>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         attr_set = true;
     }
     const uint64_t blocks = (C + kWarpsPerCta - 1) / kWarpsPerCta;
-    chunk_kernel<MODE><<<(unsigned)blocks, kWarpsPerCta * 32, smem, st>>>(in, n, g, bucket, sizes,
-                                                                         dbg);
+    chunk_kernel<MODE, SMALLW><<<(unsigned)blocks, kWarpsPerCta * 32, smem, st>>>(in, n, g, bucket, sizes, dbg);
     count_launch();
     return cudaGetLastError();
+}
+
+template <int MODE>
+cudaError_t launch_w(const uint8_t *in, uint64_t n, Geometry g, uint8_t *bucket, uint32_t *sizes,
+                     void *dbg, cudaStream_t st) {
+    return g.W <= 128 ? launch_mode<MODE, true>(in, n, g, bucket, sizes, dbg, st)
+                      : launch_mode<MODE, false>(in, n, g, bucket, sizes, dbg, st);
 }
 
 }  // namespace
@@ -512,9 +535,9 @@ cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *buck
 cudaError_t launch_chunk_kernel(int mode, const uint8_t *in, uint64_t n, Geometry g,
                                 uint8_t *bucket, uint32_t *sizes, void *dbg, cudaStream_t st) {
     switch (mode) {
-        case kModeCompress: return launch_mode<kModeCompress>(in, n, g, bucket, sizes, dbg, st);
-        case kModeDumpMatch: return launch_mode<kModeDumpMatch>(in, n, g, bucket, sizes, dbg, st);
-        default: return launch_mode<kModeDumpTokens>(in, n, g, bucket, sizes, dbg, st);
+        case kModeCompress: return launch_w<kModeCompress>(in, n, g, bucket, sizes, dbg, st);
+        case kModeDumpMatch: return launch_w<kModeDumpMatch>(in, n, g, bucket, sizes, dbg, st);
+        default: return launch_w<kModeDumpTokens>(in, n, g, bucket, sizes, dbg, st);
     }
 }
 
