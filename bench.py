@@ -29,7 +29,7 @@ import numpy as np
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-from paper_conf_cluster_ozsoys11_b200 import datagen  # noqa: E402
+from paper_conf_cluster_ozsoys11_b200 import datagen, sharding  # noqa: E402
 
 METRIC = "LZSS compress GB/s (input) at 1/2/4/8 B200 + ratio, vs CPU oracle"
 UNIT = "GB/s"
@@ -233,10 +233,17 @@ def main():
     import torch.distributed as dist
     from paper_conf_cluster_ozsoys11_b200 import culzss
 
+    # one process per GPU; BENCH_DIST_BACKEND=gloo lets several ranks share
+    # one GPU to exercise the N > 1 code path where only one GPU is visible
+    backend = os.environ.get("BENCH_DIST_BACKEND", "nccl")
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     x_np = rank_input(args.config, rank, world)
     n = int(x_np.size)
     x = torch.from_numpy(x_np).to(dev)
@@ -245,23 +252,24 @@ def main():
     out = torch.empty(culzss.max_compressed_size(n), dtype=torch.uint8, device=dev)
     payload = out[32 + 4 * C:]
     sizes = torch.empty(max(C, 1), dtype=torch.int32, device=dev)
-    totals = torch.zeros(world, dtype=torch.int64, device=dev)
-    mytotal = torch.zeros(1, dtype=torch.int64, device=dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
     stream = torch.cuda.current_stream()
     culzss.set_profiling(True)
+    placed = [None]
 
     def step():
         if world == 1:
             return culzss.compress_into(x, out), culzss.last_kernel_ms("call")
+        # rank slice -> payload + sizes; then the one exchange (NCCL all-gather
+        # of int64 totals) fixes every rank's global offsets
         t = culzss.compress_chunks(x, payload, sizes)
         ms_lib = culzss.last_kernel_ms("call")
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev0.record(stream)
-        mytotal.fill_(t)
-        dist.all_gather_into_tensor(totals, mytotal)
+        tot = sharding.exchange_totals(t, device=dev if backend == "nccl" else None)
         ev1.record(stream)
         ev1.synchronize()
+        placed[0] = sharding.placements(tot, n * world, S)[rank]
         return t, ms_lib + ev0.elapsed_time(ev1)
 
     for _ in range(args.warmup):
@@ -289,7 +297,7 @@ def main():
     clk = clocks.stop()
     total_ms = sum(step_ms)
     if world > 1:
-        t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+        t = torch.tensor([total_ms], dtype=torch.float64, device=dev if backend == "nccl" else None)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
         dist.barrier()
@@ -297,24 +305,33 @@ def main():
     # global bytes: every rank holds n bytes (weak scaling)
     n_total = n * world
     value = n_total / (ms_per_step / 1000) / 1e9
-    if world == 1:
-        stream_len = out_n
-    else:
-        stream_len = 32 + 4 * C * world + int(totals.sum().item())
+    stream_len = out_n if world == 1 else placed[0].stream_bytes
     ratio = stream_len / n_total
 
-    # roofline of the dominant kernel (fused chunk kernel): algorithmic HBM
-    # bytes = read n + write the payload (sum of sizes) + 4 B size per chunk
+    # Roofline of the dominant kernel (the fused chunk kernel, rows a1-a4) as
+    # BASELINE.json's north star defines it: the slower of (a) HBM bytes at
+    # the measured copy bandwidth and (b) the window-compare count at the
+    # integer-pipe peak.  (b): every (p, d) with 1 <= d <= min(W, p) is one
+    # byte-pair test, 516,032 per full 4 KiB chunk = 125.98 per input byte
+    # (SURVEY §8(d)), 4 tests per packed 32-bit op; peak = 148 SM x 128
+    # INT32 lanes/clk (4 SMSPs x one warp-instruction/clk) x the max SM clock
+    # (DESIGN.md §6).  The kernel searches only where the greedy parse lands,
+    # through exact hash chains, so it can beat (b); (a) is the hard floor.
     hbm_peak, sm_max_mhz, peak_kind = load_peaks()
-    pay_bytes = (out_n - 32 - 4 * C) if world == 1 else int(totals[rank].item())
-    alg_bytes = n + pay_bytes + 4 * C
+    pay_bytes = (out_n - 32 - 4 * C) if world == 1 else placed[0].payload_bytes
     ck = statistics.mean(chunk_ms)
-    achieved = alg_bytes / (ck / 1000) / 1e9
-    # context: the survey's brute-force compare roofline:
-    # 125.98 byte-pair tests per input byte at 4 per 32-bit op, against
-    # 148 SM x 128 INT32 lanes/clk x sm_max clock
+    full, tail = divmod(n, S)
+    pairs = full * (S * 128 - 128 * 129 // 2) + sum(min(128, p) for p in range(tail))
+    alg_ops = pairs / 4.0
     int_peak = 148 * 128 * sm_max_mhz * 1e6
-    t_cmp = 125.98 * n / 4 / int_peak * 1000
+    alg_bytes = n + pay_bytes + 4 * C
+    t_cmp = alg_ops / int_peak * 1000
+    t_hbm = alg_bytes / (hbm_peak * 1e9) * 1000
+    traffic = None
+    try:
+        traffic = json.load(open(os.path.join(ROOT, "profiles", "traffic.json"))).get(args.config)
+    except Exception:
+        pass
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -322,14 +339,18 @@ def main():
         "config": {"workload": f"{args.config}: {CONFIG_TEXT[args.config]}", "bytes_per_rank": n,
                    "chunk": 4096, "window": 128, "max_match": 128, "min_match": 3,
                    "l2": "flushed (256 MiB write) between steps", "parallelism": f"dp{world} (chunk ranges)",
-                   "exchange": "NCCL all_gather of per-rank compressed totals" if world > 1 else "none"},
+                   "exchange": f"{backend} all_gather of per-rank compressed totals" if world > 1 else "none"},
         "ratio": ratio,
         "kernels_ms": {"chunk": ck, "scan": statistics.mean(scan_ms), "compact": statistics.mean(compact_ms)},
-        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
-                     "frac": achieved / hbm_peak, "traffic": None, "peak_kind": peak_kind,
-                     "kernel": "chunk_kernel (fused a1-a4)", "algorithmic_bytes": alg_bytes,
-                     "alu_context": {"bruteforce_pair_tests_per_byte": 125.98, "int32_peak_tops": int_peak / 1e12,
-                                     "t_cmp_ms": t_cmp, "chunk_kernel_vs_t_cmp": t_cmp / ck}},
+        "roofline": {"bound": "alu" if t_cmp >= t_hbm else "hbm",
+                     "achieved": alg_ops / (ck / 1000) / 1e12, "peak": int_peak / 1e12, "unit": "Tops/s",
+                     "frac": max(t_cmp, t_hbm) / ck, "traffic": traffic,
+                     "kernel": "chunk_kernel (fused a1-a4)",
+                     "algorithmic": {"byte_pair_tests": pairs, "int32_ops": alg_ops, "hbm_bytes": alg_bytes},
+                     "t_cmp_ms": t_cmp, "t_hbm_ms": t_hbm, "t_kernel_ms": ck,
+                     "peak_source": "148 SM x 128 INT32 lanes/clk x %.0f MHz (DESIGN.md §6)" % sm_max_mhz,
+                     "hbm": {"achieved": alg_bytes / (ck / 1000) / 1e9, "peak": hbm_peak, "unit": "GB/s",
+                             "frac": alg_bytes / (ck / 1000) / 1e9 / hbm_peak, "peak_kind": peak_kind}},
         "clocks": clk,
         "gpu_launches": launches,
     }
@@ -350,7 +371,7 @@ def main():
                 times.append(ev0.elapsed_time(ev1))
         e2e_ms = statistics.mean(times)
         if world > 1:
-            t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
+            t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev if backend == "nccl" else None)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             e2e_ms = float(t.item())
         line["e2e"] = {"value": n_total / (e2e_ms / 1000) / 1e9, "unit": UNIT,

@@ -1,0 +1,82 @@
+"""Multi-process (gloo, CPU) test of the sharding + offset logic of SURVEY
+§8(e): R ranks compress contiguous chunk ranges (the oracle is the per-rank
+compressor here -- no GPU), all-gather their totals, and the stream
+assembled on rank 0 is byte-identical to the single-process stream."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch.multiprocessing as mp
+
+from paper_conf_cluster_ozsoys11_b200 import datagen, sharding
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, kind, n, S, out_q):
+    import torch.distributed as dist
+    import oracle as O
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        x = datagen.generate(kind, n, seed=17)  # every rank derives the same input
+        b0, b1 = sharding.byte_range(rank, world, n, S)
+        C = sharding.n_chunks(n, S)
+        c0, c1 = sharding.chunk_range(rank, world, C)
+
+        def compress_fn(sl):
+            if c1 == c0:
+                return b"", np.zeros(0, np.uint32)
+            pay, sizes = O.compress_range(x, c0, c1, S=S)
+            return pay, sizes
+
+        pay, sizes, place = sharding.compress_rank(x[b0:b1], n, rank, world, S, compress_fn)
+        assert (place.c0, place.c1) == (c0, c1)
+        stream = sharding.assemble_on_root(pay, np.asarray(sizes, "<u4").tobytes(), place, n,
+                                           (S, 128, 128, 3))
+        if rank == 0:
+            out_q.put(stream)
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,kind,n,S", [(2, "csource", 37 * 4096 + 1111, 4096),
+                                            (4, "english", 9 * 4096, 4096),
+                                            (2, "runs20", 3 * 4096 + 5, 4096),
+                                            (3, "tarmix", 5000, 1000),
+                                            (4, "random", 2 * 4096, 4096)])  # ranks with no chunks
+def test_sharded_stream_equals_single(world, kind, n, S):
+    import oracle as O
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, kind, n, S, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    stream = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    x = datagen.generate(kind, n, seed=17)
+    assert stream == O.compress(x, S=S)
+
+
+def test_placements_closed_form():
+    n, S = 10 * 4096 + 7, 4096
+    totals = [100, 0, 250, 13]
+    pl = sharding.placements(totals, n, S)
+    C = 11
+    assert [(p.c0, p.c1) for p in pl] == [(0, 2), (2, 5), (5, 8), (8, 11)]
+    assert pl[0].payload_offset == 32 + 4 * C
+    assert pl[2].payload_offset == 32 + 4 * C + 100
+    assert pl[3].table_offset == 32 + 4 * 8
+    assert all(p.stream_bytes == 32 + 4 * C + 363 for p in pl)
+    assert sharding.header(n)[:4] == b"CLZS" and len(sharding.header(n)) == 32
