@@ -52,6 +52,14 @@ constexpr uint32_t kHashMul = 0x9E3779B1u << 8;
 // 2 + (((D-1) << 8) | (L-3)) = match
 constexpr uint16_t kLit = 1;
 
+// In-word next-candidate distances for a 4-bit candidate mask z (bit j =
+// position j is a candidate): byte j = (first set bit >= j) - j, or
+// 0x80 | (4 - j) when no bit >= j is set.
+__constant__ uint32_t c_nc_tab[16] = {
+    0x81828384u, 0x81828300u, 0x81820001u, 0x81820000u, 0x81000102u, 0x81000100u, 0x81000001u,
+    0x81000000u, 0x00010203u, 0x00010200u, 0x00010001u, 0x00010000u, 0x00000102u, 0x00000100u,
+    0x00000001u, 0x00000000u};
+
 // skewed byte index of chunk position x (4 pad bytes per 128 positions)
 __device__ __forceinline__ int sk(int x) { return (int)((unsigned)x + (((unsigned)x >> 7) << 2)); }
 // skewed u16 index of position x
@@ -117,12 +125,6 @@ __device__ __forceinline__ uint16_t enc_tok(int bestL, int bestD) {
     return bestD ? (uint16_t)(2u + (((uint32_t)(bestD - 1) << 8) | (uint32_t)(bestL - 3))) : kLit;
 }
 
-__device__ __forceinline__ void mark128(uint64_t &lo, uint64_t &hi, int off) {
-    const uint64_t bit = 1ull << (off & 63);
-    lo |= off < 64 ? bit : 0ull;
-    hi |= off < 64 ? 0ull : bit;
-}
-
 // Speculative greedy walk over segment [s0, s1) from s0 as a branch-free
 // state machine: every iteration of every active lane does exactly one
 // 4-byte compare of its current candidate d at offset `off` and then updates
@@ -131,20 +133,20 @@ __device__ __forceinline__ void mark128(uint64_t &lo, uint64_t &hi, int off) {
 //     win if bytes [0, bestL] match), then its LCP 4 bytes per iteration;
 //   * a finished candidate moves to the next one on the hash chain
 //     (d += link[p-d]) or finishes the token;
-//   * a finished token is memoised in ld[], its start marked in the lane's
-//     path mask, and p jumps over candidate-free positions (literals) with
-//     nc[]; the new token's first candidate is loaded in the same iteration.
+//   * a finished token is memoised in ld[] (which also marks the path: only
+//     token starts are ever evaluated) and p jumps over candidate-free
+//     positions (literals) with nc[]; the new token's first candidate is
+//     loaded in the same iteration.
 // Returns the exit (first position >= s1 the greedy path reaches).
 __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link,
                                          const uint8_t *__restrict__ nc, uint16_t *__restrict__ ld, int m,
-                                         int W, int F, int s0, int s1, uint64_t &plo, uint64_t &phi) {
-    int p = s0 < s1 ? s0 + nc[sk(s0)] : s0;
+                                         int W, int F, int s0, int s1) {
+    int p = s0 < s1 ? min(s0 + nc[sk(s0)], s1) : s0;
     bool active = p < s1;
     int d = 0, cap = 0;
     if (active) {
         d = link[sk(p)];
         cap = min(F, m - p);
-        mark128(plo, phi, p - s0);
     }
     int k = 0, bestL = 2, bestD = 0;
     bool qr = false;
@@ -175,12 +177,11 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const 
             if (tok_done) {
                 ld[sk2(p)] = enc_tok(bestL, bestD);
                 p += bestD ? bestL : 1;
-                if (p < s1) p += nc[sk(p)];
+                if (p < s1) p = min(p + nc[sk(p)], s1);
                 active = p < s1;
                 if (active) {
                     d = link[sk(p)];
                     cap = min(F, m - p);
-                    mark128(plo, phi, p - s0);
                 }
                 bestL = 2;
                 bestD = 0;
@@ -192,36 +193,21 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const 
     return p;
 }
 
-// Re-walk from a corrected entry (fix-up rounds; short).  Reaching a token
-// start of the lane's current path (plo, phi) adopts that path's exit: the
-// greedy path from there is the same.  Tokens memoised by earlier walks cost
-// one lookup.  On return (plo, phi) is the new path, the result its exit.
+// Re-walk from a corrected entry (fix-up rounds; short).  On a lane's first
+// re-walk every memoised token start (ld != 0) belongs to its speculative
+// path, so reaching one adopts the speculative exit: the greedy path from
+// there is the same.  A later re-walk of the same lane (rare: its entry moved
+// twice) cannot tell which earlier walk a memoised start belongs to and walks
+// to the segment end, reusing memoised tokens.
 __device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link,
                         const uint8_t *__restrict__ nc, uint16_t *__restrict__ ld, int m, int W, int F, int s0,
-                        int s1, int entry, int old_exit, uint64_t &plo, uint64_t &phi) {
-    uint64_t nlo = 0, nhi = 0;
+                        int s1, int entry, int spec_exit, bool first) {
     int p = entry;
     while (true) {
-        if (p < s1) p += nc[sk(p)];
-        if (p >= s1) {
-            plo = nlo;
-            phi = nhi;
-            return p;
-        }
-        const int off = p - s0;
-        if (test128(plo, phi, off)) {  // merged: keep the old path from p on
-            if (off < 64) {
-                plo &= ~0ull << off;
-            } else {
-                plo = 0;
-                phi &= ~0ull << (off - 64);
-            }
-            plo |= nlo;
-            phi |= nhi;
-            return old_exit;
-        }
-        mark128(nlo, nhi, off);
+        if (p < s1) p = min(p + nc[sk(p)], s1);
+        if (p >= s1) return p;
         uint32_t t = ld[sk2(p)];
+        if (t && first) return spec_exit;
         if (!t) {
             t = eval_pos(cw, link, p, m, W, F);
             ld[sk2(p)] = (uint16_t)t;
@@ -364,25 +350,29 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     }
     if (s0 < s1) {
         // nc[p] = distance from p to the next candidate position (or to s1),
-        // one backward pass over the lane's link words
-        int nxt = s1;  // next candidate position after the current word
+        // one backward pass over the lane's link words: per word, the 4-bit
+        // candidate mask indexes a table of in-word distances (flag 0x80 =
+        // none in this word: 4 - j + the next word's distance)
+        int carry = 0;  // nc of the first position of the next word
 #pragma unroll 1
         for (int w = ((s1 - 1 - s0) >> 2); w >= 0; w--) {
             const int p = s0 + 4 * w;
-            const uint32_t lw = *reinterpret_cast<const uint32_t *>(link + sk(p));
-            uint32_t out = 0;
-#pragma unroll
-            for (int j = 3; j >= 0; j--) {
-                nxt = (((lw >> (8 * j)) & 0xFFu) && p + j < s1) ? p + j : nxt;
-                out |= (uint32_t)(nxt - (p + j)) << (8 * j);
-            }
+            uint32_t lw = *reinterpret_cast<const uint32_t *>(link + sk(p));
+            if (p + 4 > s1) lw &= 0xFFFFFFFFu >> (8 * (p + 4 - s1));  // positions >= s1
+            const uint32_t nz = (((lw & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | lw) & 0x80808080u;
+            const uint32_t z = (nz >> 7) * 0x10204080u >> 28;  // bit j = byte j nonzero
+            const uint32_t t = c_nc_tab[z];
+            const uint32_t flags = (t >> 7) & 0x01010101u;
+            const uint32_t out = (t & 0x7F7F7F7Fu) + flags * (uint32_t)carry;
             *reinterpret_cast<uint32_t *>(nc + sk(p)) = out;
+            carry = out & 0xFFu;
         }
     }
     __syncwarp();
-    uint64_t plo = 0, phi = 0;  // token starts (candidate positions) of the current path
-    int exitp = walk_spec(sm.cw, link, nc, ld, m, W, F, s0, s1, plo, phi);
+    const int spec_exit = walk_spec(sm.cw, link, nc, ld, m, W, F, s0, s1);
+    int exitp = spec_exit;
     int cur = s0;
+    bool first = true;
 #pragma unroll 1
     while (true) {
         int entry = __shfl_up_sync(kFull, exitp, 1);
@@ -390,7 +380,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         const bool chg = entry != cur;
         if (!__any_sync(kFull, chg)) break;
         if (chg) {
-            exitp = walk_fix(sm.cw, link, nc, ld, m, W, F, s0, s1, entry, exitp, plo, phi);
+            exitp = walk_fix(sm.cw, link, nc, ld, m, W, F, s0, s1, entry, spec_exit, first);
+            first = false;
             cur = entry;
         }
     }
@@ -426,23 +417,16 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         int p = cur;
 #pragma unroll 1
         while (p < s1) {
-            uint32_t val;
-            int nb, adv;
-            const int run = nc[sk(p)];  // candidate-free positions from p: literals
-            if (run) {
-                // up to 3 literals (27 bits) per step from one 4-byte load
-                const uint32_t w = load4(sm.cw, p);
-                const uint32_t t3 = ((w & 0xFFu) << 18) | (((w >> 8) & 0xFFu) << 9) | ((w >> 16) & 0xFFu);
-                adv = min(run, 3);
-                nb = 9 * adv;
-                val = t3 >> (27 - nb);
-            } else {
-                const uint32_t t = ld[sk2(p)];
-                const bool lit = t == kLit;
-                val = lit ? byte_at(sm.cw, p) : 0x10000u | (t - 2);
-                nb = lit ? 9 : 17;
-                adv = lit ? 1 : ((t - 2) & 0xFF) + 3;
-            }
+            // literal run (candidate-free positions), an evaluated literal, or a
+            // match; selects instead of branches
+            const int run = min((int)nc[sk(p)], s1 - p);
+            const uint32_t t = run ? (uint32_t)kLit : (uint32_t)ld[sk2(p)];
+            const int nlit = run ? min(run, 3) : (t == kLit ? 1 : 0);
+            const uint32_t w = load4(sm.cw, p);
+            const uint32_t t3 = ((w & 0xFFu) << 18) | (((w >> 8) & 0xFFu) << 9) | ((w >> 16) & 0xFFu);
+            const uint32_t val = nlit ? t3 >> (27 - 9 * nlit) : 0x10000u | (t - 2);
+            const int nb = nlit ? 9 * nlit : 17;
+            const int adv = nlit ? nlit : (int)((t - 2) & 0xFF) + 3;
             acc = (acc << nb) | val;
             nacc += nb;
             nbits += nb;
