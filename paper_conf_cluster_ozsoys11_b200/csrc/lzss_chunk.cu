@@ -54,7 +54,8 @@ constexpr uint16_t kLit = 1;
 
 // In-word next-candidate distances for a 4-bit candidate mask z (bit j =
 // position j is a candidate): byte j = (first set bit >= j) - j, or
-// 0x80 | (4 - j) when no bit >= j is set.
+// 0x80 | (4 - j) when no bit >= j is set.  Copied to shared memory per CTA:
+// lanes index it divergently, which the constant cache would serialise.
 __constant__ uint32_t c_nc_tab[16] = {
     0x81828384u, 0x81828300u, 0x81820001u, 0x81820000u, 0x81000102u, 0x81000100u, 0x81000001u,
     0x81000000u, 0x00010203u, 0x00010200u, 0x00010001u, 0x00010000u, 0x00000102u, 0x00000100u,
@@ -216,17 +217,27 @@ __device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restri
     }
 }
 
+__device__ __forceinline__ void pair_sync(int id) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(kWalkLanes) : "memory");
+}
+
 template <int MODE, bool SMALLW>
-__global__ void __launch_bounds__(kWarpsPerCta * 32, kCtasPerSm)
+__global__ void __launch_bounds__(kChunksPerCta * kWalkLanes, kCtasPerSm)
 chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__restrict__ bucket,
              uint32_t *__restrict__ sizes, void *__restrict__ dbg) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ uint32_t s_nc_tab[16];
     const int lane = threadIdx.x & 31;
-    const int wid = threadIdx.x >> 5;
-    WarpSmem &sm = reinterpret_cast<WarpSmem *>(smem_raw)[wid];
+    const int pair = threadIdx.x / kWalkLanes;     // chunk slot in the CTA
+    const int half = (threadIdx.x >> 5) & 1;       // warp within the chunk
+    const int t64 = threadIdx.x % kWalkLanes;      // walk lane 0..63
+    const int bar = 1 + pair;                      // named barrier of the warp pair
+    WarpSmem &sm = reinterpret_cast<WarpSmem *>(smem_raw)[pair];
+    if (threadIdx.x < 16) s_nc_tab[threadIdx.x] = c_nc_tab[threadIdx.x];
+    __syncthreads();
     const uint64_t C = (n + g.S - 1) / g.S;
-    const uint64_t c = (uint64_t)blockIdx.x * kWarpsPerCta + wid;
-    if (c >= C) return;  // whole warp leaves together
+    const uint64_t c = (uint64_t)blockIdx.x * kChunksPerCta + pair;
+    if (c >= C) return;  // both warps of the pair leave together
     const uint64_t start = c * g.S;
     const int m = (int)min((uint64_t)g.S, n - start);
     const int W = g.W, F = g.F;
@@ -238,20 +249,20 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     {
         uint4 *z4 = reinterpret_cast<uint4 *>(sm.cw);
         const uint4 z = make_uint4(0, 0, 0, 0);
-        for (int i = lane; i < (int)(sizeof(sm.cw) / 16); i += 32) z4[i] = z;
+        for (int i = t64; i < (int)(sizeof(sm.cw) / 16); i += kWalkLanes) z4[i] = z;
         uint4 *t4 = reinterpret_cast<uint4 *>(sm.a.u.tab);
         // u8 tables: empty = (s0 - 129) mod 256 = 0x7F (even lanes) / 0xFF (odd)
         const uint32_t e = SMALLW ? 0xFF7FFF7Fu : 0u;
         const uint4 te = make_uint4(e, e, e, e);
 #pragma unroll 4
-        for (int i = lane; i < (int)(sizeof(sm.a.u.tab) / 16); i += 32) t4[i] = te;
+        for (int i = t64; i < (int)(sizeof(sm.a.u.tab) / 16); i += kWalkLanes) t4[i] = te;
     }
-    __syncwarp();
+    pair_sync(bar);
     if ((reinterpret_cast<uintptr_t>(src) & 15) == 0) {
         // a 16-byte group never straddles a 128-position segment
         const int nvec = m >> 4;
         const uint4 *s4 = reinterpret_cast<const uint4 *>(src);
-        for (int i = lane; i < nvec; i += 32) {
+        for (int i = t64; i < nvec; i += kWalkLanes) {
             const uint4 v = __ldcs(s4 + i);
             uint32_t *d = sm.cw + (sk(i << 4) >> 2);
             d[0] = v.x;
@@ -259,79 +270,82 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
             d[2] = v.z;
             d[3] = v.w;
         }
-        for (int i = (nvec << 4) + lane; i < m; i += 32) cb[sk(i)] = src[i];
+        for (int i = (nvec << 4) + t64; i < m; i += kWalkLanes) cb[sk(i)] = src[i];
     } else {
-        for (int i = lane; i < m; i += 32) cb[sk(i)] = src[i];
+        for (int i = t64; i < m; i += kWalkLanes) cb[sk(i)] = src[i];
     }
-    __syncwarp();
-    // pad word of segment `lane` = first word of the next segment (0 past the end)
-    sm.cw[33 * lane + 32] = lane < 31 ? sm.cw[33 * (lane + 1)] : 0u;
-    __syncwarp();
+    pair_sync(bar);
+    // pad word of 128-segment `lane` = first word of the next segment (0 past the end)
+    if (half == 0) sm.cw[33 * lane + 32] = lane < 31 ? sm.cw[33 * (lane + 1)] : 0u;
+    pair_sync(bar);
 
-    // ---------------- a2 part 1: per-lane 3-gram hash chains ---------------
-    // Straight-line: every position is hashed and inserted; positions whose
-    // 3-gram would run past the chunk end (the last two) get link 0 after.
-    const int s0 = lane * kSeg;
-    const int s1 = min(s0 + kSeg, m);  // <= s0 for lanes past the chunk end
-    unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + (SMALLW ? lane : 2 * lane);
-    if (s0 < m) {
-        // the W positions before the segment (pre-insert, no links)
+    // ---------------- a2 part 1: per-lane 3-gram hash chains (warp 0) ------
+    // Lane l of warp 0 owns the 128-position build segment [128 l, 128 l + 128)
+    // and its own hash table; straight-line: every position is hashed and
+    // inserted; the last two positions (no 3-gram) get link 0 after.
+    if (half == 0) {
+        const int b0 = lane * kSeg;
+        const int b1 = min(b0 + kSeg, m);
+        unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + (SMALLW ? lane : 2 * lane);
+        if (b0 < m) {
+            // the W positions before the segment (pre-insert, no links)
 #pragma unroll 1
-        for (int q = max(0, s0 - W) & ~3; q < s0; q += 4) {
-            const uint32_t w0 = sm.cw[sk(q) >> 2], w1 = sm.cw[(sk(q) >> 2) + 1];
+            for (int q = max(0, b0 - W) & ~3; q < b0; q += 4) {
+                const uint32_t w0 = sm.cw[sk(q) >> 2], w1 = sm.cw[(sk(q) >> 2) + 1];
 #pragma unroll
-            for (int j = 0; j < 4; j++) {
-                const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
-                if (SMALLW)
-                    tabl[hash_off9(key)] = (uint8_t)(q + j);
-                else
-                    *reinterpret_cast<uint16_t *>(tabl + hash_off(key)) = (uint16_t)(q + j + kTabBias);
+                for (int j = 0; j < 4; j++) {
+                    const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
+                    if (SMALLW)
+                        tabl[hash_off9(key)] = (uint8_t)(q + j);
+                    else
+                        *reinterpret_cast<uint16_t *>(tabl + hash_off(key)) = (uint16_t)(q + j + kTabBias);
+                }
             }
-        }
-        // own segment: links
+            // own segment: links
 #pragma unroll 1
-        for (int wi = 0; wi < 4; wi++) {
-            const int pb = s0 + 32 * wi;
-            if (pb < s1) {
+            for (int wi = 0; wi < 4; wi++) {
+                const int pb = b0 + 32 * wi;
+                if (pb < b1) {
 #pragma unroll
-                for (int i = 0; i < 8; i++) {
-                    const int p = pb + 4 * i;
-                    const uint32_t w0 = sm.cw[sk(p) >> 2], w1 = sm.cw[(sk(p) >> 2) + 1];
-                    uint32_t lw = 0;
+                    for (int i = 0; i < 8; i++) {
+                        const int p = pb + 4 * i;
+                        const uint32_t w0 = sm.cw[sk(p) >> 2], w1 = sm.cw[(sk(p) >> 2) + 1];
+                        uint32_t lw = 0;
 #pragma unroll
-                    for (int j = 0; j < 4; j++) {
-                        const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
-                        uint32_t dist;
-                        if (SMALLW) {
-                            // entries hold position mod 256: every live entry is
-                            // within 256 of p, the empty value maps to 0 or > 128
-                            uint8_t *e = tabl + hash_off9(key);
-                            dist = (uint32_t)(p + j - *e) & 0xFFu;
-                            *e = (uint8_t)(p + j);
-                        } else {
-                            uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(key));
-                            dist = (uint32_t)(p + j + kTabBias) - *e;
-                            *e = (uint16_t)(p + j + kTabBias);
+                        for (int j = 0; j < 4; j++) {
+                            const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
+                            uint32_t dist;
+                            if (SMALLW) {
+                                // entries hold position mod 256: every live entry is
+                                // within 256 of p, the empty value maps to 0 or > 128
+                                uint8_t *e = tabl + hash_off9(key);
+                                dist = (uint32_t)(p + j - *e) & 0xFFu;
+                                *e = (uint8_t)(p + j);
+                            } else {
+                                uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(key));
+                                dist = (uint32_t)(p + j + kTabBias) - *e;
+                                *e = (uint16_t)(p + j + kTabBias);
+                            }
+                            lw |= (dist <= (uint32_t)W ? dist : 0u) << (8 * j);
                         }
-                        lw |= (dist <= (uint32_t)W ? dist : 0u) << (8 * j);
+                        *reinterpret_cast<uint32_t *>(link + sk(p)) = lw;
                     }
-                    *reinterpret_cast<uint32_t *>(link + sk(p)) = lw;
                 }
             }
         }
-    }
-    // positions m-2 and m-1 have no 3-gram: never candidates
+        // positions m-2 and m-1 have no 3-gram: never candidates
 #pragma unroll
-    for (int t = 1; t <= 2; t++) {
-        const int x = m - t;
-        if (x >= s0 && x < s1) link[sk(x)] = 0;
+        for (int t = 1; t <= 2; t++) {
+            const int x = m - t;
+            if (x >= b0 && x < b1) link[sk(x)] = 0;
+        }
     }
-    __syncwarp();
+    pair_sync(bar);  // tab is dead from here on
 
     if (MODE == kModeDumpMatch) {
         // every position, for per-position parity (a2)
         uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
-        for (int p = lane; p < m; p += 32) {
+        for (int p = t64; p < m; p += kWalkLanes) {
             const uint32_t t = eval_pos(sm.cw, link, p, m, W, F);
             LD[2 * p] = (uint8_t)(t == kLit ? 0 : ((t - 2) & 0xFF) + 3);
             LD[2 * p + 1] = (uint8_t)(t == kLit ? 0 : ((t - 2) >> 8) + 1);
@@ -339,14 +353,16 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         return;
     }
 
-    // ---------------- a3: lazy greedy walk, speculative per segment --------
+    // ---------------- a3: lazy greedy walk, speculative per 64-segment -----
+    const int s0 = t64 * kWSeg;
+    const int s1 = min(s0 + kWSeg, m);  // <= s0 for lanes past the chunk end
     uint8_t *nc = sm.a.u.w.nc;
     uint16_t *ld = sm.a.u.w.ld;
     {
         // zero the memoised tokens (their bytes held the hash tables)
         uint4 *l4 = reinterpret_cast<uint4 *>(ld);
         const uint4 z = make_uint4(0, 0, 0, 0);
-        for (int i = lane; i < (int)(sizeof(sm.a.u.w.ld) / 16); i += 32) l4[i] = z;
+        for (int i = t64; i < (int)(sizeof(sm.a.u.w.ld) / 16); i += kWalkLanes) l4[i] = z;
     }
     if (s0 < s1) {
         // nc[p] = distance from p to the next candidate position (or to s1),
@@ -361,31 +377,40 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
             if (p + 4 > s1) lw &= 0xFFFFFFFFu >> (8 * (p + 4 - s1));  // positions >= s1
             const uint32_t nz = (((lw & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | lw) & 0x80808080u;
             const uint32_t z = (nz >> 7) * 0x10204080u >> 28;  // bit j = byte j nonzero
-            const uint32_t t = c_nc_tab[z];
+            const uint32_t t = s_nc_tab[z];
             const uint32_t flags = (t >> 7) & 0x01010101u;
             const uint32_t out = (t & 0x7F7F7F7Fu) + flags * (uint32_t)carry;
             *reinterpret_cast<uint32_t *>(nc + sk(p)) = out;
             carry = out & 0xFFu;
         }
     }
-    __syncwarp();
+    pair_sync(bar);
     const int spec_exit = walk_spec(sm.cw, link, nc, ld, m, W, F, s0, s1);
     int exitp = spec_exit;
     int cur = s0;
     bool first = true;
+    volatile uint32_t *xf = sm.a.u.w.xfer;
 #pragma unroll 1
     while (true) {
+        // entry of walk lane t64 = exit of lane t64 - 1 (warp 1 lane 0 reads
+        // warp 0 lane 31 through shared memory)
         int entry = __shfl_up_sync(kFull, exitp, 1);
-        if (lane == 0) entry = 0;
+        if (half == 0 && lane == 31) xf[0] = (uint32_t)exitp;
+        pair_sync(bar);
+        if (lane == 0) entry = half ? (int)xf[0] : 0;
         const bool chg = entry != cur;
-        if (!__any_sync(kFull, chg)) break;
+        const bool any = __any_sync(kFull, chg);
+        if (lane == 0) xf[1 + half] = any;
+        pair_sync(bar);
+        const bool go = xf[1] | xf[2];
+        pair_sync(bar);  // xf is reused by the next round
+        if (!go) break;
         if (chg) {
             exitp = walk_fix(sm.cw, link, nc, ld, m, W, F, s0, s1, entry, spec_exit, first);
             first = false;
             cur = entry;
         }
     }
-    __syncwarp();
 
     if (MODE == kModeDumpTokens) {
         uint32_t *tok = reinterpret_cast<uint32_t *>(dbg) + start;
@@ -403,13 +428,14 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         }
         return;
     }
+    pair_sync(bar);  // link is dead: staging may overwrite it
 
     // ---------------- a4: bit-pack ----------------------------------------
-    // Each lane emits its path's tokens MSB-first into its own staging words
-    // starting at bit 0 (one token per loop iteration; a token is a literal,
-    // a pair of literals of a candidate-free run, or a match); after the warp
-    // scan of bit counts the staged words are shifted into place.
-    uint32_t *stage = reinterpret_cast<uint32_t *>(sm.a.link) + lane * kStageWords;  // link is dead
+    // Each walk lane emits its path's tokens MSB-first into its own staging
+    // words starting at bit 0 (a token is up to 3 literals of a candidate-free
+    // run, an evaluated literal, or a match); after the scan of bit counts the
+    // staged words are shifted into place.
+    uint32_t *stage = reinterpret_cast<uint32_t *>(sm.a.link) + t64 * kStageWords;
     int nbits = 0;
     {
         uint64_t acc = 0;
@@ -417,8 +443,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         int p = cur;
 #pragma unroll 1
         while (p < s1) {
-            // literal run (candidate-free positions), an evaluated literal, or a
-            // match; selects instead of branches
+            // selects instead of branches
             const int run = min((int)nc[sk(p)], s1 - p);
             const uint32_t t = run ? (uint32_t)kLit : (uint32_t)ld[sk2(p)];
             const int nlit = run ? min(run, 3) : (t == kLit ? 1 : 0);
@@ -438,19 +463,25 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         }
         if (nacc > 0) stage[nw] = (uint32_t)(acc << (32 - nacc));
     }
+    // exclusive scan of bit counts over the 64 walk lanes
     int incl = nbits;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
         const int y = __shfl_up_sync(kFull, incl, o);
         if (lane >= o) incl += y;
     }
+    if (half == 0 && lane == 31) xf[0] = (uint32_t)incl;
+    pair_sync(bar);
+    const int w0tot = (int)xf[0];
+    if (half) incl += w0tot;
     const int excl = incl - nbits;
-    const int total = __shfl_sync(kFull, incl, 31);
+    if (half == 1 && lane == 31) xf[1] = (uint32_t)incl;
+    pair_sync(bar);
+    const int total = (int)xf[1];
     const int nwords = (total + 31) >> 5;
     uint32_t *ow = reinterpret_cast<uint32_t *>(ld);  // ld is dead: payload words
-    __syncwarp();
-    for (int i = lane; i < nwords + 1; i += 32) ow[i] = 0;
-    __syncwarp();
+    for (int i = t64; i < nwords + 1; i += kWalkLanes) ow[i] = 0;
+    pair_sync(bar);
     {
         // shift the lane's staged words to bit offset excl; output words shared
         // with the neighbouring lanes (first, last, spill) are OR-ed atomically
@@ -470,14 +501,14 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
             if (o) atomicOr(&ow[base + nsw], o);
         }
     }
-    __syncwarp();
+    pair_sync(bar);
 
     // payload -> bucket c (bytes in stream order: big-endian words)
     const int nbytes = (total + 7) >> 3;
     const uint64_t stride = bucket_stride(g.S);
     uint4 *dst = reinterpret_cast<uint4 *>(bucket + c * stride);
     const uint4 *o4 = reinterpret_cast<const uint4 *>(ow);
-    for (int i = lane; i < (nbytes + 15) >> 4; i += 32) {
+    for (int i = t64; i < (nbytes + 15) >> 4; i += kWalkLanes) {
         uint4 v = o4[i];
         v.x = __byte_perm(v.x, 0, 0x0123);
         v.y = __byte_perm(v.y, 0, 0x0123);
@@ -485,7 +516,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         v.w = __byte_perm(v.w, 0, 0x0123);
         dst[i] = v;
     }
-    if (lane == 0) sizes[c] = (uint32_t)nbytes;
+    if (t64 == 0) sizes[c] = (uint32_t)nbytes;
 }
 
 template <int MODE, bool SMALLW>
@@ -493,7 +524,7 @@ cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *buck
                         uint32_t *sizes, void *dbg, cudaStream_t st) {
     const uint64_t C = (n + g.S - 1) / g.S;
     if (C == 0) return cudaSuccess;
-    const size_t smem = sizeof(WarpSmem) * kWarpsPerCta;
+    const size_t smem = sizeof(WarpSmem) * kChunksPerCta;
     static bool attr_set = false;  // benign race: idempotent
     if (!attr_set) {
         cudaError_t e = cudaFuncSetAttribute(chunk_kernel<MODE, SMALLW>,
@@ -501,8 +532,9 @@ cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *buck
         if (e != cudaSuccess) return e;
         attr_set = true;
     }
-    const uint64_t blocks = (C + kWarpsPerCta - 1) / kWarpsPerCta;
-    chunk_kernel<MODE, SMALLW><<<(unsigned)blocks, kWarpsPerCta * 32, smem, st>>>(in, n, g, bucket, sizes, dbg);
+    const uint64_t blocks = (C + kChunksPerCta - 1) / kChunksPerCta;
+    chunk_kernel<MODE, SMALLW><<<(unsigned)blocks, kChunksPerCta * kWalkLanes, smem, st>>>(in, n, g, bucket,
+                                                                                            sizes, dbg);
     count_launch();
     return cudaGetLastError();
 }
