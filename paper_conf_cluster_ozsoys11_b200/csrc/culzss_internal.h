@@ -14,7 +14,7 @@ constexpr int kSeg = 128;           // positions per lane segment (32 x 128 = 40
 constexpr int kHashBits = 8;        // per-lane 3-gram hash table, W > 128: 256 u16 heads
 constexpr int kHashBitsSmallW = 9;  // W <= 128: 512 u8 heads (relative positions)
 constexpr int kChunksPerCta = 3;    // chunks per CTA
-constexpr int kWarpsPerChunk = 2;   // warp 0 builds the hash chains; both warps walk
+constexpr int kWarpsPerChunk = 2;   // warp 0 builds the hash chains; all warps walk
 constexpr int kWalkLanes = 32 * kWarpsPerChunk;   // 64 walk segments per chunk
 constexpr int kWSeg = kChunkMax / kWalkLanes;     // 64 positions per walk segment
 constexpr int kCtasPerSm = 3;
@@ -33,11 +33,10 @@ struct Geometry {
 // memoised tokens (`ld`).  After the walks link/nc become per-lane bit
 // staging and `ld` the packed payload words.
 constexpr int kSkewBytes = kChunkMax + 4 * (kChunkMax / kSeg);   // 4224
-// per-walk-lane bit staging: a 64-position segment emits at most 9 bits per
-// position (a 17-bit match covers >= 3 positions) + one 17-bit token crossing
-// its end: 593 bits = 19 words
-constexpr int kStageWords = 19;                      // odd stride: conflict-free
-constexpr int kStagePad = kWalkLanes * kStageWords * 4 - kSkewBytes;   // 640
+// per-walk-lane bit staging: a segment emits at most 9 bits per position (a
+// 17-bit match covers >= 3 positions) + one 17-bit token crossing its end
+constexpr int kStageWords = ((kWSeg * 9 + 17 + 31) / 32) | 1;   // odd stride: conflict-free
+constexpr int kStagePad = (kWalkLanes * kStageWords * 4 > kSkewBytes ? kWalkLanes * kStageWords * 4 - kSkewBytes : 0) + 16;
 struct __align__(16) WarpSmem {
     uint32_t cw[(kSkewBytes + 16) / 4];              // chunk bytes (skewed) + zero tail
     struct {
@@ -47,7 +46,7 @@ struct __align__(16) WarpSmem {
                                                      // or u8 position mod 256, 512 buckets (W <= 128)
             struct {
                 uint8_t pad[kStagePad];              // staging = link + pad (after the walks)
-                uint32_t xfer[4];                    // cross-warp exchange (exits, flags, bit counts)
+                uint32_t xfer[8];                    // cross-warp exchange (exits, flags, bit counts)
                 uint8_t nc[kSkewBytes];              // distance to next candidate position (<= s1)
                 uint16_t ld[kChunkMax + 2 * (kChunkMax / kSeg)];  // memoised token (0 = not evaluated)
             } w;

@@ -229,7 +229,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     __shared__ uint32_t s_nc_tab[16];
     const int lane = threadIdx.x & 31;
     const int pair = threadIdx.x / kWalkLanes;     // chunk slot in the CTA
-    const int half = (threadIdx.x >> 5) & 1;       // warp within the chunk
+    const int half = (threadIdx.x >> 5) % kWarpsPerChunk;  // warp within the chunk
     const int t64 = threadIdx.x % kWalkLanes;      // walk lane 0..63
     const int bar = 1 + pair;                      // named barrier of the warp pair
     WarpSmem &sm = reinterpret_cast<WarpSmem *>(smem_raw)[pair];
@@ -395,14 +395,17 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         // entry of walk lane t64 = exit of lane t64 - 1 (warp 1 lane 0 reads
         // warp 0 lane 31 through shared memory)
         int entry = __shfl_up_sync(kFull, exitp, 1);
-        if (half == 0 && lane == 31) xf[0] = (uint32_t)exitp;
+        if (lane == 31) xf[half] = (uint32_t)exitp;
         pair_sync(bar);
-        if (lane == 0) entry = half ? (int)xf[0] : 0;
+        if (lane == 0) entry = half ? (int)xf[half - 1] : 0;
         const bool chg = entry != cur;
         const bool any = __any_sync(kFull, chg);
-        if (lane == 0) xf[1 + half] = any;
+        pair_sync(bar);  // all reads of xf done
+        if (lane == 0) xf[half] = any;
         pair_sync(bar);
-        const bool go = xf[1] | xf[2];
+        bool go = false;
+#pragma unroll
+        for (int k = 0; k < kWarpsPerChunk; k++) go |= xf[k] != 0;
         pair_sync(bar);  // xf is reused by the next round
         if (!go) break;
         if (chg) {
@@ -470,14 +473,17 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         const int y = __shfl_up_sync(kFull, incl, o);
         if (lane >= o) incl += y;
     }
-    if (half == 0 && lane == 31) xf[0] = (uint32_t)incl;
+    if (lane == 31) xf[half] = (uint32_t)incl;
     pair_sync(bar);
-    const int w0tot = (int)xf[0];
-    if (half) incl += w0tot;
+    int before = 0, total = 0;
+#pragma unroll
+    for (int k = 0; k < kWarpsPerChunk; k++) {
+        const int v = (int)xf[k];
+        before += k < half ? v : 0;
+        total += v;
+    }
+    incl += before;
     const int excl = incl - nbits;
-    if (half == 1 && lane == 31) xf[1] = (uint32_t)incl;
-    pair_sync(bar);
-    const int total = (int)xf[1];
     const int nwords = (total + 31) >> 5;
     uint32_t *ow = reinterpret_cast<uint32_t *>(ld);  // ld is dead: payload words
     for (int i = t64; i < nwords + 1; i += kWalkLanes) ow[i] = 0;
