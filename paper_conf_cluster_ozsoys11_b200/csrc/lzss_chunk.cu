@@ -142,11 +142,16 @@ __device__ __forceinline__ uint16_t enc_tok(int bestL, int bestD) {
 __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link,
                                          const uint8_t *__restrict__ nc, uint16_t *__restrict__ ld, int m,
                                          int W, int F, int s0, int s1) {
-    int p = s0 < s1 ? min(s0 + nc[sk(s0)], s1) : s0;
+    // token starts stay inside the lane's segment, which never crosses a
+    // 128-position skew boundary: p-indexed arrays use a constant offset
+    const int so = (s0 >> 7) << 2;
+    const uint8_t *ncs = nc + so, *lks = link + so;
+    uint16_t *lds = ld + (so >> 1);
+    int p = s0 < s1 ? min(s0 + ncs[s0], s1) : s0;
     bool active = p < s1;
     int d = 0, cap = 0;
     if (active) {
-        d = link[sk(p)];
+        d = lks[p];
         cap = min(F, m - p);
     }
     int k = 0, bestL = 2, bestD = 0;
@@ -176,12 +181,12 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const 
                 qr = bestL >= 3;
             }
             if (tok_done) {
-                ld[sk2(p)] = enc_tok(bestL, bestD);
+                lds[p] = enc_tok(bestL, bestD);
                 p += bestD ? bestL : 1;
-                if (p < s1) p = min(p + nc[sk(p)], s1);
+                if (p < s1) p = min(p + ncs[p], s1);
                 active = p < s1;
                 if (active) {
-                    d = link[sk(p)];
+                    d = lks[p];
                     cap = min(F, m - p);
                 }
                 bestL = 2;
@@ -370,17 +375,18 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         // candidate mask indexes a table of in-word distances (flag 0x80 =
         // none in this word: 4 - j + the next word's distance)
         int carry = 0;  // nc of the first position of the next word
+        const int so = (s0 >> 7) << 2;  // constant skew inside the segment
 #pragma unroll 1
         for (int w = ((s1 - 1 - s0) >> 2); w >= 0; w--) {
             const int p = s0 + 4 * w;
-            uint32_t lw = *reinterpret_cast<const uint32_t *>(link + sk(p));
+            uint32_t lw = *reinterpret_cast<const uint32_t *>(link + so + p);
             if (p + 4 > s1) lw &= 0xFFFFFFFFu >> (8 * (p + 4 - s1));  // positions >= s1
             const uint32_t nz = (((lw & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | lw) & 0x80808080u;
             const uint32_t z = (nz >> 7) * 0x10204080u >> 28;  // bit j = byte j nonzero
             const uint32_t t = s_nc_tab[z];
             const uint32_t flags = (t >> 7) & 0x01010101u;
             const uint32_t out = (t & 0x7F7F7F7Fu) + flags * (uint32_t)carry;
-            *reinterpret_cast<uint32_t *>(nc + sk(p)) = out;
+            *reinterpret_cast<uint32_t *>(nc + so + p) = out;
             carry = out & 0xFFu;
         }
     }
@@ -444,13 +450,20 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         uint64_t acc = 0;
         int nacc = 0, nw = 0;
         int p = cur;
+        // all positions read here lie in the lane's segment (+3 bytes into the
+        // pad word): constant skew offsets
+        const int so = (s0 >> 7) << 2;
+        const uint8_t *ncs = nc + so;
+        const uint16_t *lds = ld + (so >> 1);
+        const uint8_t *cbs = cb + so;
 #pragma unroll 1
         while (p < s1) {
             // selects instead of branches
-            const int run = min((int)nc[sk(p)], s1 - p);
-            const uint32_t t = run ? (uint32_t)kLit : (uint32_t)ld[sk2(p)];
+            const int run = min((int)ncs[p], s1 - p);
+            const uint32_t t = run ? (uint32_t)kLit : (uint32_t)lds[p];
             const int nlit = run ? min(run, 3) : (t == kLit ? 1 : 0);
-            const uint32_t w = load4(sm.cw, p);
+            const int a = so + p;
+            const uint32_t w = __funnelshift_r(sm.cw[a >> 2], sm.cw[(a >> 2) + 1], (a & 3) * 8);
             const uint32_t t3 = ((w & 0xFFu) << 18) | (((w >> 8) & 0xFFu) << 9) | ((w >> 16) & 0xFFu);
             const uint32_t val = nlit ? t3 >> (27 - 9 * nlit) : 0x10000u | (t - 2);
             const int nb = nlit ? 9 * nlit : 17;
