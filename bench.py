@@ -53,6 +53,7 @@ def parse_args():
     ap.add_argument("--config", default="c2_csource_128m", choices=sorted(datagen.CONFIGS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-decompress", action="store_true")
     return ap.parse_args()
 
 
@@ -354,7 +355,29 @@ def main():
         "clocks": clk,
         "gpu_launches": launches,
     }
-    # e2e through the public API with host buffers (pinned), N=1 only per rank
+    # a6: decompression of this rank's stream (N=1: the full stream), device
+    # time of the decode kernel and of the whole culzss_decompress call
+    if world == 1 and not args.no_decompress:
+        dec = torch.empty(n, dtype=torch.uint8, device=dev)
+        sview = out[:out_n]
+        dms, cms = [], []
+        for it in range(args.warmup + args.steps):
+            flush.fill_(1)
+            torch.cuda.synchronize()
+            ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            ev0.record(stream)
+            culzss.decompress(sview, dec)
+            ev1.record(stream)
+            ev1.synchronize()
+            if it >= args.warmup:
+                dms.append(culzss.last_kernel_ms("decode"))
+                cms.append(ev0.elapsed_time(ev1))
+        ok = bool(torch.equal(dec, x))
+        line["decompress"] = {"value": n / (statistics.mean(cms) / 1000) / 1e9, "unit": "GB/s (output)",
+                              "decode_kernel_ms": statistics.mean(dms), "call_ms": statistics.mean(cms),
+                              "roundtrip_exact": ok}
+        del dec
+
     if not args.no_e2e:
         hin = torch.from_numpy(x_np).pin_memory()
         hout = torch.empty(culzss.max_compressed_size(n), dtype=torch.uint8).pin_memory()
