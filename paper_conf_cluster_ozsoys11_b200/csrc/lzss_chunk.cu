@@ -68,10 +68,12 @@ __device__ __forceinline__ int sk2(int x) { return x + ((x >> 7) << 1); }
 
 __device__ __forceinline__ uint32_t load4(const uint32_t *cw, int x) {
     // bytes x..x+3 of the chunk (little endian), from two aligned words; the
-    // pad word after each segment repeats the next segment's first word
-    const int a = sk(x);
-    const uint32_t lo = cw[a >> 2], hi = cw[(a >> 2) + 1];
-    return __funnelshift_r(lo, hi, (a & 3) * 8);
+    // pad word after each segment repeats the next segment's first word.
+    // Word index of sk(x) = x/4 + x/128; the funnel shift masks its amount to
+    // 5 bits, so 8x selects the byte offset within the word.
+    const unsigned ux = (unsigned)x;
+    const unsigned wi = (ux >> 2) + (ux >> 7);
+    return __funnelshift_r(cw[wi], cw[wi + 1], ux << 3);
 }
 
 __device__ __forceinline__ uint32_t byte_at(const uint32_t *cw, int x) {
