@@ -470,8 +470,9 @@ culzss_status culzss_decompress(const void *in, size_t in_n, void *out, size_t *
     const uint64_t offs_off = (C * 4 + 255) / 256 * 256;
     const uint64_t ws_off = offs_off + (C * 8 + 255) / 256 * 256;
     const uint64_t tot_off = ws_off + (scan_workspace_words(C) * 8 + 255) / 256 * 256;
+    const uint64_t tb_off = tot_off + 256;
     Workspace ws(st);
-    CK(ws.alloc(tot_off + 256));
+    CK(ws.alloc(tb_off + decode_scratch_bytes(C)));
     uint8_t *base = static_cast<uint8_t *>(ws.p);
     uint32_t *sizes = reinterpret_cast<uint32_t *>(base + tab_off);
     uint64_t *offsets = reinterpret_cast<uint64_t *>(base + offs_off);
@@ -490,7 +491,7 @@ culzss_status culzss_decompress(const void *in, size_t in_n, void *out, size_t *
     t_prof.reset();
     t_prof.rec(1, st);
     CK(launch_decode(src + 32 + 4 * C, sizes, offsets, C, n, g, static_cast<uint8_t *>(out),
-                     err, st));
+                     err, reinterpret_cast<uint32_t *>(base + tb_off), st));
     t_prof.rec(2, st);
     CK(cudaMemcpyAsync(hw, err, 4, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
