@@ -449,36 +449,41 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     uint32_t *stage = reinterpret_cast<uint32_t *>(sm.a.link) + t64 * kStageWords;
     int nbits = 0;
     {
+        // Uniform position scan (no token jumps): every position >= the lane's
+        // true entry is either inside a path match (covered) or a path token
+        // start; a token start's memoised ld[] is its token whichever walk
+        // wrote it, and is 0 for candidate-free positions (literals).  Each
+        // position emits 0, 9 or 17 bits.
         uint64_t acc = 0;
         int nacc = 0, nw = 0;
-        int p = cur;
-        // all positions read here lie in the lane's segment (+3 bytes into the
-        // pad word): constant skew offsets
+        int cov = cur;  // positions < cov are covered (by the previous lane or a match)
         const int so = (s0 >> 7) << 2;
-        const uint8_t *ncs = nc + so;
-        const uint16_t *lds = ld + (so >> 1);
-        const uint8_t *cbs = cb + so;
+        const uint32_t *ldw = reinterpret_cast<const uint32_t *>(ld + (so >> 1) + s0);  // 2 tokens / word
+        const uint32_t *cbw = reinterpret_cast<const uint32_t *>(cb + so + s0);         // 4 bytes / word
+        const int ng = (s1 - s0 + 3) >> 2;
 #pragma unroll 1
-        while (p < s1) {
-            // selects instead of branches
-            const int run = min((int)ncs[p], s1 - p);
-            const uint32_t t = run ? (uint32_t)kLit : (uint32_t)lds[p];
-            const int nlit = run ? min(run, 3) : (t == kLit ? 1 : 0);
-            const int a = so + p;
-            const uint32_t w = __funnelshift_r(sm.cw[a >> 2], sm.cw[(a >> 2) + 1], (a & 3) * 8);
-            const uint32_t t3 = ((w & 0xFFu) << 18) | (((w >> 8) & 0xFFu) << 9) | ((w >> 16) & 0xFFu);
-            const uint32_t val = nlit ? t3 >> (27 - 9 * nlit) : 0x10000u | (t - 2);
-            const int nb = nlit ? 9 * nlit : 17;
-            const int adv = nlit ? nlit : (int)((t - 2) & 0xFF) + 3;
-            acc = (acc << nb) | val;
-            nacc += nb;
-            nbits += nb;
-            p += adv;
-            if (nacc >= 32) {
-                nacc -= 32;
-                stage[nw++] = (uint32_t)(acc >> nacc);
+        for (int i = max(0, (cov - s0) >> 2); i < ng; i = max(i + 1, (cov - s0) >> 2)) {
+            // groups wholly inside a match are skipped
+            const uint32_t bytes = cbw[i];
+            const uint32_t t01 = ldw[2 * i], t23 = ldw[2 * i + 1];
+#pragma unroll
+            for (int j = 0; j < 4; j++) {
+                const int p = s0 + 4 * i + j;
+                const uint32_t t = (j < 2 ? t01 : t23) >> (16 * (j & 1)) & 0xFFFFu;
+                const bool on = p >= cov && p < s1;
+                const bool mt = on && t >= 2;
+                const int nb = mt ? 17 : (on ? 9 : 0);
+                const uint32_t val = mt ? 0x10000u | (t - 2) : (bytes >> (8 * j)) & 0xFFu;
+                cov = mt ? p + (int)((t - 2) & 0xFF) + 3 : cov;
+                acc = (acc << nb) | (nb ? val : 0u);
+                nacc += nb;
+                if (nacc >= 32) {
+                    nacc -= 32;
+                    stage[nw++] = (uint32_t)(acc >> nacc);
+                }
             }
         }
+        nbits = 32 * nw + nacc;
         if (nacc > 0) stage[nw] = (uint32_t)(acc << (32 - nacc));
     }
     // exclusive scan of bit counts over the 64 walk lanes
