@@ -29,14 +29,15 @@ struct Geometry {
 // word of a segment duplicates the first word of the next one, so an
 // unaligned 4-byte load is two aligned word loads anywhere in the chunk.
 // During the chain build `tab` holds the per-lane hash heads; afterwards the
-// same bytes hold nc[] (distance to the next candidate position) and the
-// memoised tokens (`ld`).  After the walks link/nc become per-lane bit
+// same bytes hold the memoised tokens (`ld`) and an unskewed copy of the
+// chunk for the walks.  After the walks link (+ pad) becomes per-lane bit
 // staging and `ld` the packed payload words.
 constexpr int kSkewBytes = kChunkMax + 4 * (kChunkMax / kSeg);   // 4224
 // per-walk-lane bit staging: a segment emits at most 9 bits per position (a
 // 17-bit match covers >= 3 positions) + one 17-bit token crossing its end
 constexpr int kStageWords = ((kWSeg * 9 + 17 + 31) / 32) | 1;   // odd stride: conflict-free
 constexpr int kStagePad = (kWalkLanes * kStageWords * 4 > kSkewBytes ? kWalkLanes * kStageWords * 4 - kSkewBytes : 0) + 16;
+constexpr int kUcwWords = kChunkMax / 4 + 4;  // + zero tail: 8-byte loads read 3 words
 struct __align__(16) WarpSmem {
     uint32_t cw[(kSkewBytes + 16) / 4];              // chunk bytes (skewed) + zero tail
     struct {
@@ -47,15 +48,16 @@ struct __align__(16) WarpSmem {
             struct {
                 uint8_t pad[kStagePad];              // staging = link + pad (after the walks)
                 uint32_t xfer[8];                    // cross-warp exchange (exits, flags, bit counts)
-                uint8_t nc[kSkewBytes];              // distance to next candidate position (<= s1)
                 uint16_t ld[kChunkMax + 2 * (kChunkMax / kSeg)];  // memoised token (0 = not evaluated)
+                uint32_t ucw[kUcwWords];             // unskewed chunk copy for the walks' 8-byte compares
+                                                     // (random access: the skew buys nothing there)
             } w;
         } u;
     } a;
 };
 static_assert(sizeof(WarpSmem) <= 24848, "smem layout");
-static_assert(offsetof(WarpSmem, a.u.w.nc) - offsetof(WarpSmem, a.link) >= kWalkLanes * kStageWords * 4,
-              "staging (over link + pad) must not reach nc");
+static_assert(offsetof(WarpSmem, a.u.w.xfer) - offsetof(WarpSmem, a.link) >= kWalkLanes * kStageWords * 4,
+              "staging (over link + pad) must not reach xfer / ld");
 static_assert((kChunkMax * 9 / 8 + 16) <= sizeof(WarpSmem::a.u.w.ld), "payload words fit in ld");
 
 __host__ __device__ inline uint64_t bucket_stride(uint32_t S) { return (((uint64_t)S * 9 + 7) / 8 + 15) / 16 * 16; }

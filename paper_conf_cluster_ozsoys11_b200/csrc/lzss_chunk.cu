@@ -48,18 +48,9 @@ namespace {
 constexpr uint32_t kFull = 0xffffffffu;
 constexpr uint32_t kTabBias = 0x1000;   // table entry = position + bias; 0 = empty
 constexpr uint32_t kHashMul = 0x9E3779B1u << 8;
-// memoised token encoding in ld[]: 0 = not evaluated, 1 = literal,
-// 2 + (((D-1) << 8) | (L-3)) = match
-constexpr uint16_t kLit = 1;
-
-// In-word next-candidate distances for a 4-bit candidate mask z (bit j =
-// position j is a candidate): byte j = (first set bit >= j) - j, or
-// 0x80 | (4 - j) when no bit >= j is set.  Copied to shared memory per CTA:
-// lanes index it divergently, which the constant cache would serialise.
-__constant__ uint32_t c_nc_tab[16] = {
-    0x81828384u, 0x81828300u, 0x81820001u, 0x81820000u, 0x81000102u, 0x81000100u, 0x81000001u,
-    0x81000000u, 0x00010203u, 0x00010200u, 0x00010001u, 0x00010000u, 0x00000102u, 0x00000100u,
-    0x00000001u, 0x00000000u};
+// memoised token encoding in ld[]: 0 = not evaluated, 2 = literal,
+// (D << 8) | (L - 3) = match (>= 0x100; L - 3 fits 8 bits for F <= 258)
+constexpr uint16_t kLit = 2;
 
 // skewed byte index of chunk position x (4 pad bytes per 128 positions)
 __device__ __forceinline__ int sk(int x) { return (int)((unsigned)x + (((unsigned)x >> 7) << 2)); }
@@ -76,8 +67,36 @@ __device__ __forceinline__ uint32_t load4(const uint32_t *cw, int x) {
     return __funnelshift_r(cw[wi], cw[wi + 1], ux << 3);
 }
 
-__device__ __forceinline__ uint32_t byte_at(const uint32_t *cw, int x) {
-    return reinterpret_cast<const uint8_t *>(cw)[sk(x)];
+// The walks compare on an unskewed, byte-swapped (big-endian words) copy of
+// the chunk: bytes x..x+7 are two funnel shifts of three aligned words with
+// byte x in the most significant position, so the number of equal leading
+// bytes of two such values is a count of leading zeros of their XOR.
+struct Be8 {
+    uint32_t hi, lo;  // bytes x..x+3, x+4..x+7
+};
+__device__ __forceinline__ Be8 load8(const uint32_t *__restrict__ u, int x) {
+    const uint32_t *w = u + ((unsigned)x >> 2);
+    const uint32_t a = w[0], b = w[1], c = w[2];
+    const unsigned sh = (unsigned)x << 3;  // the funnel shift masks it to 5 bits
+    return Be8{__funnelshift_l(b, a, sh), __funnelshift_l(c, b, sh)};
+}
+
+// first candidate position >= p of the lane's segment [s0, s1), or s1 (p if
+// p >= s1 already).  rc0 / rc1: candidate bits of positions s0..s0+31 /
+// s0+32..s0+63, position s0+i at bit 31-i (reversed: next = count of
+// leading zeros)
+__device__ __forceinline__ int next_cand(uint32_t rc0, uint32_t rc1, int p, int s0, int s1) {
+    if (p >= s1) return p;
+    const int o = p - s0;  // < 64
+    const int sh = o & 31;
+    const uint32_t r0 = rc0 << sh;
+    const int n0 = r0 ? o + __clz(r0) : 32 + __clz(rc1);
+    const int n1 = o + __clz(rc1 << sh);  // clz(0) = 32: past the segment
+    return min(s0 + (o < 32 ? n0 : n1), s1);
+}
+
+__device__ __forceinline__ bool is_cand(uint32_t rc0, uint32_t rc1, int o) {
+    return ((o < 32 ? rc0 : rc1) << (o & 31)) >> 31;
 }
 
 // byte offset (into the per-lane-interleaved table) of the 3-gram hash of a
@@ -87,11 +106,7 @@ __device__ __forceinline__ uint32_t hash_off(uint32_t w) { return ((w * kHashMul
 // W <= 128 variant: 9-bit hash, u8 entries [h][lane] at byte 32 h + lane
 __device__ __forceinline__ uint32_t hash_off9(uint32_t w) { return ((w * kHashMul) >> 18) & 0x3FE0u; }
 
-__device__ __forceinline__ int tok_len(uint32_t t) { return t == kLit ? 1 : ((t - 2) & 0xFF) + 3; }
-
-__device__ __forceinline__ bool test128(uint64_t lo, uint64_t hi, int off) {
-    return ((off < 64 ? lo >> off : hi >> (off - 64)) & 1ull) != 0;
-}
+__device__ __forceinline__ int tok_len(uint32_t t) { return t >= 0x100 ? (int)(t & 0xFF) + 3 : 1; }
 
 // Token at one position by a plain chain walk (debug entry point only).
 __device__ uint32_t eval_pos(const uint32_t *cw, const uint8_t *link, int p, int m, int W, int F) {
@@ -121,35 +136,31 @@ __device__ uint32_t eval_pos(const uint32_t *cw, const uint8_t *link, int p, int
         if (!l2 || d + l2 > W) break;
         d += l2;
     }
-    return bestD ? 2u + (((uint32_t)(bestD - 1) << 8) | (uint32_t)(bestL - 3)) : kLit;
-}
-
-__device__ __forceinline__ uint16_t enc_tok(int bestL, int bestD) {
-    return bestD ? (uint16_t)(2u + (((uint32_t)(bestD - 1) << 8) | (uint32_t)(bestL - 3))) : kLit;
+    return bestD ? ((uint32_t)bestD << 8) | (uint32_t)(bestL - 3) : kLit;
 }
 
 // Speculative greedy walk over segment [s0, s1) from s0 as a branch-free
 // state machine: every iteration of every active lane does exactly one
-// 4-byte compare of its current candidate d at offset `off` and then updates
-// its state with selects:
-//   * a candidate first gets a reject test at offset bestL-3 (it can only
-//     win if bytes [0, bestL] match), then its LCP 4 bytes per iteration;
+// 8-byte compare of its current candidate d at offset `off` (on the unskewed
+// chunk copy u) and then updates its state with selects:
+//   * a candidate first gets a 4-byte reject test at offset bestL-3 (it can
+//     only win if bytes [0, bestL] match), then its LCP 8 bytes per iteration;
 //   * a finished candidate moves to the next one on the hash chain
 //     (d += link[p-d]) or finishes the token;
-//   * a finished token is memoised in ld[] (which also marks the path: only
-//     token starts are ever evaluated) and p jumps over candidate-free
-//     positions (literals) with nc[]; the new token's first candidate is
-//     loaded in the same iteration.
+//   * a finished token is memoised in ld[] and p jumps over candidate-free
+//     positions (literals) with the lane's candidate mask; the new token's
+//     first candidate is loaded in the same iteration.
 // Returns the exit (first position >= s1 the greedy path reaches).
-__device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link,
-                                         const uint8_t *__restrict__ nc, uint16_t *__restrict__ ld, int m,
-                                         int W, int F, int s0, int s1) {
+__device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const uint8_t *__restrict__ link,
+                                         uint32_t rc0, uint32_t rc1, uint16_t *__restrict__ ld, int m, int W,
+                                         int F, int s0,
+                                         int s1) {
     // token starts stay inside the lane's segment, which never crosses a
     // 128-position skew boundary: p-indexed arrays use a constant offset
     const int so = (s0 >> 7) << 2;
-    const uint8_t *ncs = nc + so, *lks = link + so;
+    const uint8_t *lks = link + so;
     uint16_t *lds = ld + (so >> 1);
-    int p = s0 < s1 ? min(s0 + ncs[s0], s1) : s0;
+    int p = next_cand(rc0, rc1, s0, s0, s1);
     bool active = p < s1;
     int d = 0, cap = 0;
     if (active) {
@@ -164,15 +175,16 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const 
             const int q = p - d;
             const int off = qr ? bestL - 3 : k;
             const int lq = link[sk(q)];  // next chain member, loaded with the compare words
-            const uint32_t x = load4(cw, q + off) ^ load4(cw, p + off);
-            const int fb = x ? (__ffs(x) - 1) >> 3 : 4;
-            const bool cand_done = qr ? (x != 0) : (x != 0 || k + 4 >= cap);
+            const Be8 vq = load8(u, q + off), vp = load8(u, p + off);
+            const uint32_t xh = vq.hi ^ vp.hi, xl = vq.lo ^ vp.lo;
+            const int fb = xh ? __clz(xh) >> 3 : 4 + (__clz(xl) >> 3);  // equal leading bytes (<= 8)
+            const bool cand_done = qr ? xh != 0 : (fb < 8 || k + 8 >= cap);
             const int L = min(k + fb, cap);
             const bool upd = !qr && cand_done && L > bestL;
             bestL = upd ? L : bestL;
             bestD = upd ? d : bestD;
-            k = qr ? 0 : k + 4;
-            qr = qr && x != 0;
+            k = qr ? 0 : k + 8;
+            qr = qr && xh != 0;
             bool tok_done = false;
             if (cand_done) {
                 const int l2 = bestL == cap ? 0 : lq;
@@ -183,9 +195,8 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const 
                 qr = bestL >= 3;
             }
             if (tok_done) {
-                lds[p] = enc_tok(bestL, bestD);
-                p += bestD ? bestL : 1;
-                if (p < s1) p = min(p + ncs[p], s1);
+                lds[p] = (uint16_t)(bestD ? (bestD << 8) | (bestL - 3) : kLit);
+                p = next_cand(rc0, rc1, p + (bestD ? bestL : 1), s0, s1);
                 active = p < s1;
                 if (active) {
                     d = lks[p];
@@ -207,12 +218,12 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ cw, const 
 // there is the same.  A later re-walk of the same lane (rare: its entry moved
 // twice) cannot tell which earlier walk a memoised start belongs to and walks
 // to the segment end, reusing memoised tokens.
-__device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link,
-                        const uint8_t *__restrict__ nc, uint16_t *__restrict__ ld, int m, int W, int F, int s0,
-                        int s1, int entry, int spec_exit, bool first) {
+__device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link, uint32_t rc0, uint32_t rc1,
+                        uint16_t *__restrict__ ld, int m, int W, int F, int s0, int s1, int entry,
+                        int spec_exit, bool first) {
     int p = entry;
     while (true) {
-        if (p < s1) p = min(p + nc[sk(p)], s1);
+        p = next_cand(rc0, rc1, p, s0, s1);
         if (p >= s1) return p;
         uint32_t t = ld[sk2(p)];
         if (t && first) return spec_exit;
@@ -233,15 +244,12 @@ __global__ void __launch_bounds__(kChunksPerCta * kWalkLanes, kCtasPerSm)
 chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__restrict__ bucket,
              uint32_t *__restrict__ sizes, void *__restrict__ dbg) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ uint32_t s_nc_tab[16];
     const int lane = threadIdx.x & 31;
     const int pair = threadIdx.x / kWalkLanes;     // chunk slot in the CTA
     const int half = (threadIdx.x >> 5) % kWarpsPerChunk;  // warp within the chunk
     const int t64 = threadIdx.x % kWalkLanes;      // walk lane 0..63
     const int bar = 1 + pair;                      // named barrier of the warp pair
     WarpSmem &sm = reinterpret_cast<WarpSmem *>(smem_raw)[pair];
-    if (threadIdx.x < 16) s_nc_tab[threadIdx.x] = c_nc_tab[threadIdx.x];
-    __syncthreads();
     const uint64_t C = (n + g.S - 1) / g.S;
     const uint64_t c = (uint64_t)blockIdx.x * kChunksPerCta + pair;
     if (c >= C) return;  // both warps of the pair leave together
@@ -354,8 +362,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
         for (int p = t64; p < m; p += kWalkLanes) {
             const uint32_t t = eval_pos(sm.cw, link, p, m, W, F);
-            LD[2 * p] = (uint8_t)(t == kLit ? 0 : ((t - 2) & 0xFF) + 3);
-            LD[2 * p + 1] = (uint8_t)(t == kLit ? 0 : ((t - 2) >> 8) + 1);
+            LD[2 * p] = (uint8_t)(t == kLit ? 0 : (t & 0xFF) + 3);
+            LD[2 * p + 1] = (uint8_t)(t == kLit ? 0 : t >> 8);
         }
         return;
     }
@@ -363,37 +371,37 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     // ---------------- a3: lazy greedy walk, speculative per 64-segment -----
     const int s0 = t64 * kWSeg;
     const int s1 = min(s0 + kWSeg, m);  // <= s0 for lanes past the chunk end
-    uint8_t *nc = sm.a.u.w.nc;
     uint16_t *ld = sm.a.u.w.ld;
+    uint32_t *ucw = sm.a.u.w.ucw;
     {
-        // zero the memoised tokens (their bytes held the hash tables)
+        // zero the memoised tokens (their bytes held the hash tables) and
+        // unskew the chunk for the walks' compares
         uint4 *l4 = reinterpret_cast<uint4 *>(ld);
         const uint4 z = make_uint4(0, 0, 0, 0);
         for (int i = t64; i < (int)(sizeof(sm.a.u.w.ld) / 16); i += kWalkLanes) l4[i] = z;
+        for (int j = t64; j < kUcwWords; j += kWalkLanes) ucw[j] = __byte_perm(sm.cw[j + (j >> 5)], 0, 0x0123);
     }
+    // candidate mask: bit i = position s0 + i (< s1) has a chain link
+    uint32_t rc0 = 0, rc1 = 0;
     if (s0 < s1) {
-        // nc[p] = distance from p to the next candidate position (or to s1),
-        // one backward pass over the lane's link words: per word, the 4-bit
-        // candidate mask indexes a table of in-word distances (flag 0x80 =
-        // none in this word: 4 - j + the next word's distance)
-        int carry = 0;  // nc of the first position of the next word
         const int so = (s0 >> 7) << 2;  // constant skew inside the segment
-#pragma unroll 1
-        for (int w = ((s1 - 1 - s0) >> 2); w >= 0; w--) {
-            const int p = s0 + 4 * w;
-            uint32_t lw = *reinterpret_cast<const uint32_t *>(link + so + p);
-            if (p + 4 > s1) lw &= 0xFFFFFFFFu >> (8 * (p + 4 - s1));  // positions >= s1
+        uint32_t h[2] = {0, 0};
+#pragma unroll
+        for (int w = 0; w < kWSeg / 4; w++) {
+            const uint32_t lw = *reinterpret_cast<const uint32_t *>(link + so + s0 + 4 * w);
             const uint32_t nz = (((lw & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | lw) & 0x80808080u;
-            const uint32_t z = (nz >> 7) * 0x10204080u >> 28;  // bit j = byte j nonzero
-            const uint32_t t = s_nc_tab[z];
-            const uint32_t flags = (t >> 7) & 0x01010101u;
-            const uint32_t out = (t & 0x7F7F7F7Fu) + flags * (uint32_t)carry;
-            *reinterpret_cast<uint32_t *>(nc + so + p) = out;
-            carry = out & 0xFFu;
+            h[w >> 3] |= ((nz >> 7) * 0x10204080u >> 28) << (4 * (w & 7));  // bit j = byte j nonzero
         }
+        if (s1 - s0 < 64) {  // positions >= s1 (garbage links)
+            const int r = s1 - s0;
+            h[0] &= r >= 32 ? 0xFFFFFFFFu : (1u << r) - 1;
+            h[1] &= r <= 32 ? 0u : (1u << (r - 32)) - 1;
+        }
+        rc0 = __brev(h[0]);
+        rc1 = __brev(h[1]);
     }
     pair_sync(bar);
-    const int spec_exit = walk_spec(sm.cw, link, nc, ld, m, W, F, s0, s1);
+    const int spec_exit = walk_spec(ucw, link, rc0, rc1, ld, m, W, F, s0, s1);
     int exitp = spec_exit;
     int cur = s0;
     bool first = true;
@@ -417,7 +425,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         pair_sync(bar);  // xf is reused by the next round
         if (!go) break;
         if (chg) {
-            exitp = walk_fix(sm.cw, link, nc, ld, m, W, F, s0, s1, entry, spec_exit, first);
+            exitp = walk_fix(sm.cw, link, rc0, rc1, ld, m, W, F, s0, s1, entry, spec_exit, first);
             first = false;
             cur = entry;
         }
@@ -428,12 +436,12 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         for (int p = s0; p < s1; p++) tok[p] = 0;
         int p = cur;
         while (p < s1) {
-            if (nc[sk(p)]) {
+            if (!is_cand(rc0, rc1, p - s0)) {
                 tok[p] = 1;
                 p++;
             } else {
                 const uint32_t t = ld[sk2(p)];
-                tok[p] = t == kLit ? 1u : ((uint32_t)(((t - 2) & 0xFF) + 3) << 16) | (((t - 2) >> 8) + 1);
+                tok[p] = t == kLit ? 1u : (((t & 0xFF) + 3) << 16) | (t >> 8);
                 p += tok_len(t);
             }
         }
@@ -471,10 +479,10 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                 const int p = s0 + 4 * i + j;
                 const uint32_t t = (j < 2 ? t01 : t23) >> (16 * (j & 1)) & 0xFFFFu;
                 const bool on = p >= cov && p < s1;
-                const bool mt = on && t >= 2;
+                const bool mt = on && t >= 0x100;
                 const int nb = mt ? 17 : (on ? 9 : 0);
-                const uint32_t val = mt ? 0x10000u | (t - 2) : (bytes >> (8 * j)) & 0xFFu;
-                cov = mt ? p + (int)((t - 2) & 0xFF) + 3 : cov;
+                const uint32_t val = mt ? t + (0x10000u - 0x100u) : (bytes >> (8 * j)) & 0xFFu;  // 1|D-1|L-3
+                cov = mt ? p + (int)(t & 0xFF) + 3 : cov;
                 acc = (acc << nb) | (nb ? val : 0u);
                 nacc += nb;
                 if (nacc >= 32) {

@@ -3,7 +3,7 @@
 # one ncu --set full capture of the fused chunk kernel.  Usage: tools/gpu_round.sh TAG
 TAG=${1:-x}
 cd "${GRAFT_REPO_ROOT:-$(dirname "$0")/..}"
-timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -8
+timeout 240 python -m pytest tests -m gpu -x -q 2>&1 | tail -8
 python bench.py --steps 10 --warmup 3 --no-cpu-baseline > gpurun_out/bench_c2_$TAG.json 2>&1
 python bench.py --config c4_random_1g --steps 5 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/bench_c4_$TAG.json 2>&1
 python bench.py --config c3_runs20_1g --steps 5 --warmup 3 --no-cpu-baseline --no-e2e > gpurun_out/bench_c3_$TAG.json 2>&1
