@@ -9,9 +9,12 @@
 
 #include <atomic>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
+#include <vector>
+#include <algorithm>
 
 #include "../../include/culzss.h"
 #include "culzss_internal.h"
@@ -171,24 +174,35 @@ void prof_finish_compress() {
     t_times.call = t_prof.between(0, 5);
 }
 
+// Workspace of compress_core for C chunks: bucket | sizes | offsets | scan ws
+struct CoreLayout {
+    uint64_t sizes_off, offs_off, ws_off, total;
+    CoreLayout(uint64_t C, uint32_t S) {
+        const uint64_t bucket_bytes = C * bucket_stride(S) + 16;
+        sizes_off = (bucket_bytes + 255) / 256 * 256;
+        offs_off = sizes_off + (C * 4 + 255) / 256 * 256;
+        ws_off = offs_off + (C * 8 + 255) / 256 * 256;
+        total = ws_off + scan_workspace_words(C) * 8;
+    }
+};
+
 // Core compression of n bytes at device `in` into: payload region `pay`
 // (capacity checked by callers), table `table` (may be null), total payload
 // bytes -> device word `dev_total`.  Sizes go to `sizes` (device, C words).
+// `wsp`: a CoreLayout-sized device workspace, or null to allocate one on st.
 culzss_status compress_core(const uint8_t *in, uint64_t n, const Geometry &g, uint8_t *pay,
                             uint32_t *table, uint32_t *sizes_out, uint64_t *dev_total,
-                            cudaStream_t st) {
+                            cudaStream_t st, void *wsp = nullptr) {
     const uint64_t C = n_chunks(n, g.S);
     const uint64_t stride = bucket_stride(g.S);
-    const uint64_t scan_ws = scan_workspace_words(C);
-    // workspace: bucket | sizes | offsets | scan ws
-    const uint64_t bucket_bytes = C * stride + 16;
-    const uint64_t sizes_off = (bucket_bytes + 255) / 256 * 256;
-    const uint64_t offs_off = sizes_off + (C * 4 + 255) / 256 * 256;
-    const uint64_t ws_off = offs_off + (C * 8 + 255) / 256 * 256;
-    const uint64_t total_bytes = ws_off + scan_ws * 8;
+    const CoreLayout lay(C, g.S);
+    const uint64_t sizes_off = lay.sizes_off, offs_off = lay.offs_off, ws_off = lay.ws_off;
     Workspace ws(st);
-    CK(ws.alloc(total_bytes));
-    uint8_t *base = static_cast<uint8_t *>(ws.p);
+    if (!wsp) {
+        CK(ws.alloc(lay.total));
+        wsp = ws.p;
+    }
+    uint8_t *base = static_cast<uint8_t *>(wsp);
     uint8_t *bucket = base;
     uint32_t *sizes = sizes_out ? sizes_out : reinterpret_cast<uint32_t *>(base + sizes_off);
     uint64_t *offsets = reinterpret_cast<uint64_t *>(base + offs_off);
@@ -370,6 +384,51 @@ culzss_status culzss_compress_chunks(const void *in_slice, size_t slice_n, void 
     return s;
 }
 
+// Pipelined host-memory compression: the chunks go in groups of ~8 MiB.
+// Group k's H2D, fused kernel, scan and compaction (into its own staging
+// region) run on compute stream k % 3, so the H2D of one group overlaps the
+// kernels of the previous ones; its size table goes straight to its final
+// host position.  Its payload's host position needs the totals of all
+// earlier groups: the scan writes each group total into mapped host memory
+// (no copy-engine round trip), the host waits for group k-2 (the GPU has
+// groups k-1 and k queued) and issues that payload's D2H on its own stream.
+namespace {
+constexpr int kPipeStreams = 3;
+struct HostPipe {
+    cudaStream_t cs[kPipeStreams] = {}, ds = {};
+    cudaEvent_t ev_in = {};
+    std::vector<cudaEvent_t> ev;
+    uint64_t *htot = nullptr;  // mapped pinned: the scan kernel writes group totals here
+    uint64_t *dtot = nullptr;  // its device alias
+    size_t htot_n = 0;
+    bool ok = false;
+    bool init(size_t groups) {
+        if (!ok) {
+            for (auto &c : cs)
+                if (cudaStreamCreateWithFlags(&c, cudaStreamNonBlocking) != cudaSuccess) return false;
+            if (cudaStreamCreateWithFlags(&ds, cudaStreamNonBlocking) != cudaSuccess ||
+                cudaEventCreateWithFlags(&ev_in, cudaEventDisableTiming) != cudaSuccess)
+                return false;
+            ok = true;
+        }
+        while (ev.size() < groups) {
+            cudaEvent_t e;
+            if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return false;
+            ev.push_back(e);
+        }
+        if (htot_n < groups) {
+            if (htot) cudaFreeHost(htot);
+            htot = nullptr;
+            if (cudaHostAlloc(&htot, groups * 8, cudaHostAllocMapped) != cudaSuccess) return false;
+            if (cudaHostGetDevicePointer(&dtot, htot, 0) != cudaSuccess) return false;
+            htot_n = groups;
+        }
+        return true;
+    }
+};
+thread_local HostPipe t_pipe;
+}  // namespace
+
 culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host, size_t *out_n,
                                    const culzss_params *p, culzss_stream_t stream) {
     lib_init();
@@ -379,24 +438,114 @@ culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host
     culzss_status s = check_params(p, &g);
     if (s != CULZSS_OK) return s;
     const uint64_t C = n_chunks(n, g.S);
+    if (C > 0xFFFFFFFFull) return CULZSS_ERR_INVALID_ARG;
     const uint64_t bound = 32 + 4 * C + payload_bound(n, g.S);
     if (*out_n < bound) {
         *out_n = (size_t)bound;
         return CULZSS_ERR_BUFFER_TOO_SMALL;
     }
     cudaStream_t st = (cudaStream_t)stream;
-    Workspace ws(st);
+    static const uint64_t group_bytes = [] {  // CULZSS_GROUP_KB: pipeline tuning knob
+        const char *e = getenv("CULZSS_GROUP_KB");
+        const long v = e ? atol(e) : 0;
+        return v > 0 ? (uint64_t)v << 10 : (8ull << 20);
+    }();
+    const uint64_t gc = std::max<uint64_t>(1, group_bytes / g.S);  // chunks per group
+    const uint64_t G = (C + gc - 1) / gc;
+    if (G <= 1) {  // one group: no overlap to gain
+        Workspace ws(st);
+        const uint64_t in_bytes = (n + 255) / 256 * 256;
+        CK(ws.alloc(in_bytes + bound));
+        uint8_t *din = static_cast<uint8_t *>(ws.p);
+        uint8_t *dout = din + in_bytes;
+        if (n) CK(cudaMemcpyAsync(din, in_host, n, cudaMemcpyHostToDevice, st));
+        size_t on = (size_t)bound;
+        s = culzss_compress(din, n, dout, &on, p, stream);
+        if (s != CULZSS_OK) return s;
+        CK(cudaMemcpyAsync(out_host, dout, on, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        *out_n = on;
+        return CULZSS_OK;
+    }
+    HostPipe &hp = t_pipe;
+    if (!hp.init(G)) return cuda_fail(cudaErrorMemoryAllocation);
+    // device: input | header + table (contiguous, as in the stream) | per-group
+    // staging at its worst-case offset | group totals | two core workspaces
+    const CoreLayout lay(gc, g.S);
     const uint64_t in_bytes = (n + 255) / 256 * 256;
-    CK(ws.alloc(in_bytes + bound));
+    const uint64_t ht_bytes = (32 + 4 * C + 255) / 256 * 256;
+    const uint64_t stg_bytes = (payload_bound(n, g.S) + 255) / 256 * 256;
+    const uint64_t core_bytes = (lay.total + 255) / 256 * 256;
+    Workspace ws(st);
+    CK(ws.alloc(in_bytes + ht_bytes + stg_bytes + kPipeStreams * core_bytes));
     uint8_t *din = static_cast<uint8_t *>(ws.p);
-    uint8_t *dout = din + in_bytes;
-    if (n) CK(cudaMemcpyAsync(din, in_host, n, cudaMemcpyHostToDevice, st));
-    size_t on = (size_t)bound;
-    s = culzss_compress(din, n, dout, &on, p, stream);
-    if (s != CULZSS_OK) return s;
-    CK(cudaMemcpyAsync(out_host, dout, on, cudaMemcpyDeviceToHost, st));
+    uint8_t *dht = din + in_bytes;
+    uint8_t *dstg = dht + ht_bytes;
+    uint8_t *dcore = dstg + stg_bytes;
+    uint8_t *hout = static_cast<uint8_t *>(out_host);
+    const uint8_t *hin = static_cast<const uint8_t *>(in_host);
+    struct Drain {  // on an error return, no internal stream may still use ws
+        HostPipe &hp;
+        bool done = false;
+        ~Drain() {
+            if (done) return;
+            for (auto cs : hp.cs) cudaStreamSynchronize(cs);
+            cudaStreamSynchronize(hp.ds);
+            cudaGetLastError();
+        }
+    } drain{hp};
+    t_prof.reset();
+    t_prof.rec(0, st);
+    CK(launch_header(dht, n, g, st));
+    CK(cudaEventRecord(hp.ev_in, st));  // the workspace and header exist
+    for (auto cs : hp.cs) CK(cudaStreamWaitEvent(cs, hp.ev_in, 0));
+    CK(cudaStreamWaitEvent(hp.ds, hp.ev_in, 0));
+    CK(cudaMemcpyAsync(hout, dht, 32, cudaMemcpyDeviceToHost, hp.ds));
+    uint64_t base = 0;  // payload bytes of the groups whose D2H is issued
+    auto issue_payload = [&](uint64_t k) -> culzss_status {
+        CK(cudaEventSynchronize(hp.ev[k]));
+        const uint64_t t = hp.htot[k];
+        if (t) {
+            CK(cudaStreamWaitEvent(hp.ds, hp.ev[k], 0));
+            CK(cudaMemcpyAsync(hout + 32 + 4 * C + base, dstg + payload_bound(k * gc * g.S, g.S), t,
+                               cudaMemcpyDeviceToHost, hp.ds));
+        }
+        base += t;
+        return CULZSS_OK;
+    };
+    for (uint64_t k = 0; k < G; k++) {
+        cudaStream_t cs = hp.cs[k % kPipeStreams];
+        const uint64_t c0 = k * gc, c1 = std::min(C, c0 + gc);
+        const uint64_t b0 = c0 * g.S, nb = std::min<uint64_t>(n, c1 * g.S) - b0;
+        CK(cudaMemcpyAsync(din + b0, hin + b0, nb, cudaMemcpyHostToDevice, cs));
+        s = compress_core(din + b0, nb, g, dstg + payload_bound(b0, g.S),
+                          reinterpret_cast<uint32_t *>(dht + 32) + c0, nullptr, hp.dtot + k, cs,
+                          dcore + (k % kPipeStreams) * core_bytes);
+        if (s != CULZSS_OK) return s;
+        CK(cudaMemcpyAsync(hout + 32 + 4 * c0, dht + 32 + 4 * c0, 4 * (c1 - c0), cudaMemcpyDeviceToHost,
+                           cs));
+        CK(cudaEventRecord(hp.ev[k], cs));
+        if (k >= 2) {
+            s = issue_payload(k - 2);
+            if (s != CULZSS_OK) return s;
+        }
+    }
+    for (uint64_t k = G >= 2 ? G - 2 : 0; k < G; k++) {
+        s = issue_payload(k);
+        if (s != CULZSS_OK) return s;
+    }
+    // the caller's stream resumes after everything (the workspace is freed on it)
+    CK(cudaEventRecord(hp.ev_in, hp.ds));
+    CK(cudaStreamWaitEvent(st, hp.ev_in, 0));
+    for (auto cs : hp.cs) {
+        CK(cudaEventRecord(hp.ev[0], cs));
+        CK(cudaStreamWaitEvent(st, hp.ev[0], 0));
+    }
+    t_prof.rec(5, st);
     CK(cudaStreamSynchronize(st));
-    *out_n = on;
+    drain.done = true;
+    if (t_profiling) t_times.call = t_prof.between(0, 5);
+    *out_n = (size_t)(32 + 4 * C + base);
     return CULZSS_OK;
 }
 

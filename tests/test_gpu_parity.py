@@ -230,6 +230,32 @@ def test_compress_host_matches(env):
     assert culzss.compress_host(x[:0]).tobytes() == O.compress(x[:0])
 
 
+@pytest.mark.parametrize("kind,n", [("csource", (8 << 20) + 1), ("tarmix", 3 * (8 << 20) + 4097 * 3 + 17),
+                                    ("random", 2 * (8 << 20)), ("runs20", 5 * (8 << 20) - 1)])
+def test_compress_host_pipelined(env, kind, n):
+    """Inputs above one 8 MiB group take the pipelined host path (groups on
+    two compute streams, payload D2H placed by the earlier groups' totals):
+    the host stream equals the device-API stream, whose chunks the oracle
+    checks (first, last, and a spread of sampled chunks)."""
+    torch, culzss = env
+    x = datagen.generate(kind, n, seed=21)
+    h = culzss.compress_host(x).tobytes()
+    d = culzss.compress(dev(torch, x)).cpu().numpy().tobytes()
+    assert h == d
+    S, C = 4096, (n + 4095) // 4096
+    sizes = np.frombuffer(h[32:32 + 4 * C], "<u4").astype(np.int64)
+    offs = np.concatenate([[0], np.cumsum(sizes)]) + 32 + 4 * C
+    for c in sorted({0, C - 1} | set(range(0, C, max(1, C // 24)))):
+        ref = O.compress(x[c * S:min(n, (c + 1) * S)])
+        assert h[offs[c]:offs[c + 1]] == ref[36:], c
+    # pinned host buffers through the raw-pointer entry point (bench e2e path)
+    xin = torch.from_numpy(x).pin_memory()
+    cap = culzss.max_compressed_size(n)
+    out = torch.empty(cap, dtype=torch.uint8).pin_memory()
+    on = culzss.compress_host_ptr(xin.data_ptr(), n, out.data_ptr(), cap)
+    assert out[:on].numpy().tobytes() == h
+
+
 def test_sharded_assembly_equals_single(env):
     """SURVEY §8(e) on one GPU: R simulated ranks compress chunk ranges with
     culzss_compress_chunks; placing table slices at 32 + 4*c0 and payloads
