@@ -98,6 +98,31 @@ def test_stream_params_variants(env, S, W, F):
         assert gpu_stream(env, x, S=S, W=W, F=F) == O.compress(x, S=S, W=W, F=F), kind
 
 
+@pytest.mark.parametrize("S,W,F", [(4096, 1, 3), (4096, 255, 258), (4096, 16, 18), (1, 128, 128),
+                                   (100, 7, 9), (129, 3, 5), (1000, 128, 128), (4000, 100, 250)])
+def test_decoder_params_variants(env, S, W, F):
+    """Row a6 on oracle streams of every parameter shape (lane spans vs chunk size)."""
+    torch, culzss = env
+    for kind in ("english", "runs20", "period20", "random"):
+        x = datagen.generate(kind, 30011, seed=S + 1)
+        s = O.compress(x, S=S, W=W, F=F)
+        y = culzss.decompress(dev(torch, np.frombuffer(s, np.uint8)))
+        assert y.cpu().numpy().tobytes() == x.tobytes(), kind
+
+
+def test_decoder_unaligned_input_and_output(env):
+    torch, culzss = env
+    x = datagen.generate("csource", 70001, seed=9)
+    s = np.frombuffer(O.compress(x), np.uint8)
+    for ioff in (0, 1, 3, 7, 13):
+        buf = torch.zeros(s.size + 32, dtype=torch.uint8, device="cuda")
+        buf[ioff:ioff + s.size] = dev(torch, s)
+        for oo in (0, 1, 2, 5):
+            out = torch.zeros(x.size + 8, dtype=torch.uint8, device="cuda")
+            culzss.decompress(buf[ioff:ioff + s.size], out[oo:oo + x.size])
+            assert out[oo:oo + x.size].cpu().numpy().tobytes() == x.tobytes(), (ioff, oo)
+
+
 @pytest.mark.parametrize("kind", ["english", "csource", "runs20", "period20", "random", "tarmix"])
 def test_match_search_per_position(env, kind):
     """Row a2: (L, D) at every position of several chunks + a ragged tail."""

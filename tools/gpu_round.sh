@@ -13,5 +13,5 @@ if [ -z "$NO_NCU" ]; then
       > gpurun_out/prof_$TAG.log 2>&1
 fi
 for f in gpurun_out/bench_c*_$TAG.json; do
-  python -c "import json,sys; d=json.loads(open(sys.argv[1]).read().strip().splitlines()[-1]); print(sys.argv[1], round(d['value'],1), {k: round(v,3) for k,v in d['kernels_ms'].items()}, round(d['ratio'],4))" $f
+  python -c "import json,sys; d=json.loads(open(sys.argv[1]).read().strip().splitlines()[-1]); print(sys.argv[1], round(d['value'],1), {k: round(v,3) for k,v in d['kernels_ms'].items()}, round(d['ratio'],4), 'dec', round(d.get('decompress',{}).get('value',0),1), round(d.get('decompress',{}).get('decode_kernel_ms',0),3))" $f
 done
