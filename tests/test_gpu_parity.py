@@ -279,6 +279,10 @@ def test_compress_host_pipelined(env, kind, n):
     out = torch.empty(cap, dtype=torch.uint8).pin_memory()
     on = culzss.compress_host_ptr(xin.data_ptr(), n, out.data_ptr(), cap)
     assert out[:on].numpy().tobytes() == h
+    # device-placed payloads land at any byte alignment of the pinned output
+    out2 = torch.zeros(cap + 8, dtype=torch.uint8).pin_memory()
+    on = culzss.compress_host_ptr(xin.data_ptr(), n, out2.data_ptr() + 3, cap)
+    assert out2[3:3 + on].numpy().tobytes() == h
 
 
 def test_sharded_assembly_equals_single(env):
