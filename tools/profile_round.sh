@@ -21,7 +21,7 @@ for cfg in c2_csource_128m c4_random_1g c3_runs20_1g; do
       -o gpurun_out/full_${cfg}_$TAG python bench.py --config $cfg --steps 1 --warmup 1 --no-cpu-baseline --no-e2e \
       > /dev/null 2>&1
 done
-for k in boundary_kernel decode_kernel; do
+for k in walk_kernel decode_kernel; do
   ncu --set full --clock-control none --import-source on -k regex:$k -s 1 -c 1 \
       -o gpurun_out/full_${k}_c2_$TAG python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-e2e \
       > /dev/null 2>&1
