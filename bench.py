@@ -40,7 +40,8 @@ CONFIG_TEXT = {
     "c2_csource_128m": "128 MiB source-code-like text (csource generator, seed 2; PAPER.md:1@23843 'C files')",
     "c3_runs20_1g": "1 GiB runs of 20 identical bytes (runs20 generator, seed 3; PAPER.md:1@24662)",
     "c4_random_1g": "1 GiB random bytes (splitmix64, seed 4)",
-    "c5_tarmix_64g": "64 GiB tarball-like mix (tarmix generator, seed 5) -- per-rank slices",
+    "c5_tarmix_64g": "64 GiB tarball-like mix (tarmix generator, seed 5) -- per-rank slices; at N=1 the "
+                     "8 GiB slice of rank 0 of a dp8 split (64 GiB + its output + buckets exceed one GPU)",
 }
 
 
@@ -71,7 +72,7 @@ def rank_input(cfg: str, rank: int, world: int) -> np.ndarray:
     spec = datagen.CONFIGS[cfg]
     n = spec["n"]
     if cfg == "c5_tarmix_64g":
-        n = n // world
+        n = n // (world if world > 1 else 8)
     seed = spec["seed"] + 1000 * rank
     return datagen.generate(spec["kind"], n, seed)
 
