@@ -634,12 +634,10 @@ culzss_status culzss_decompress(const void *in, size_t in_n, void *out, size_t *
     CK(launch_scan(sizes, C, offsets, total, scanws, st));
     uint64_t *hw = host_word();
     if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
-    CK(cudaMemcpyAsync(hw, total, 8, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    if (32 + 4 * C + hw[0] != in_n) return CULZSS_ERR_CORRUPT;
+    // the walk kernel checks the table against the payload length (no sync here)
     t_prof.reset();
     t_prof.rec(1, st);
-    CK(launch_decode(src + 32 + 4 * C, sizes, offsets, C, n, g, static_cast<uint8_t *>(out),
+    CK(launch_decode(src + 32 + 4 * C, in_n - 32 - 4 * C, sizes, offsets, C, n, g, static_cast<uint8_t *>(out),
                      err, reinterpret_cast<uint32_t *>(base + tb_off), st));
     t_prof.rec(2, st);
     CK(cudaMemcpyAsync(hw, err, 4, cudaMemcpyDeviceToHost, st));

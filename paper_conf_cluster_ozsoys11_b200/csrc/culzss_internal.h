@@ -75,7 +75,7 @@ cudaError_t launch_compact(const uint8_t *bucket, uint64_t stride, const uint32_
                            const uint64_t *offsets, uint64_t C, uint8_t *out_payload,
                            uint32_t *out_table, cudaStream_t st);
 cudaError_t launch_header(uint8_t *out, uint64_t n, Geometry g, cudaStream_t st);
-cudaError_t launch_decode(const uint8_t *payload, const uint32_t *sizes,
+cudaError_t launch_decode(const uint8_t *payload, uint64_t pay_len, const uint32_t *sizes,
                           const uint64_t *offsets, uint64_t C, uint64_t n, Geometry g,
                           uint8_t *out, uint32_t *err, uint32_t *tb_scratch, cudaStream_t st);
 uint64_t decode_scratch_bytes(uint64_t C);
