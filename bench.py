@@ -55,6 +55,8 @@ def parse_args():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-decompress", action="store_true")
+    ap.add_argument("--no-versions", action="store_true",
+                    help="skip timing params.version = 2 (the paper's V2 all-position search) beside the default")
     return ap.parse_args()
 
 
@@ -356,6 +358,34 @@ def main():
         "clocks": clk,
         "gpu_launches": launches,
     }
+    # params.version = 2 (the paper's V2 search design: every position, every
+    # window offset) on the same input, same protocol, fewer
+    # steps: the measured cost of the brute-force design the default replaces
+    if world == 1 and not args.no_versions:
+        p2 = culzss.Params.make(version=2)
+        out2 = torch.empty_like(out)
+        v2_ms, v2_ck = [], []
+        n2 = 0
+        for it in range(1 + max(1, min(3, args.steps))):
+            flush.fill_(1)
+            torch.cuda.synchronize()
+            n2 = culzss.compress_into(x, out2, p2)
+            if it >= 1:
+                v2_ms.append(culzss.last_kernel_ms("call"))
+                v2_ck.append(culzss.last_kernel_ms("chunk"))
+        ck2 = statistics.mean(v2_ck)
+        line["versions"] = {
+            "0": {"what": "lazy greedy search over 3-gram hash chains (default)", "value": value,
+                  "chunk_ms": ck, "roofline_frac": max(t_cmp, t_hbm) / ck},
+            "2": {"what": "paper V2 design: warp-cooperative longest match at every position over all "
+                          "window offsets, __reduce_max_sync argmax",
+                  "value": n / (statistics.mean(v2_ms) / 1000) / 1e9, "unit": UNIT, "chunk_ms": ck2,
+                  "compares_tops": alg_ops / (ck2 / 1000) / 1e12, "roofline_frac": max(t_cmp, t_hbm) / ck2,
+                  "steps": len(v2_ms),
+                  "stream_identical": bool(n2 == out_n and torch.equal(out2[:n2], out[:out_n]))},
+        }
+        del out2
+
     # a6: decompression of this rank's stream (N=1: the full stream), device
     # time of the decode kernel and of the whole culzss_decompress call
     if world == 1 and not args.no_decompress:

@@ -78,8 +78,9 @@ culzss_status check_params(const culzss_params *p, Geometry *g) {
     if (p->min_match != 3 || p->chunk_size < 1 || p->window < 1 || p->window > 256 ||
         p->max_match < 3 || p->max_match > 258 || p->reserved != 0)
         return CULZSS_ERR_INVALID_ARG;
-    if (p->version != 0 || p->chunk_size > (uint32_t)kChunkMax || p->window > 255)
+    if ((p->version != 0 && p->version != 2) || p->chunk_size > (uint32_t)kChunkMax || p->window > 255)
         return CULZSS_ERR_UNSUPPORTED;
+    g->V = p->version;
     g->S = p->chunk_size;
     g->W = p->window;
     g->F = p->max_match;

@@ -21,6 +21,8 @@ constexpr int kCtasPerSm = 3;
 
 struct Geometry {
     uint32_t S, W, F;               // chunk, window, max match (MIN is 3)
+    uint32_t V = 0;                 // kernel version: 0 = lazy hash-chain search,
+                                    // 2 = the paper's V2 all-position search
 };
 
 // Per-warp shared memory.  Per-position arrays use a SKEWED layout: 4 pad

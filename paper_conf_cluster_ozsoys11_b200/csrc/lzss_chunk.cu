@@ -235,11 +235,67 @@ __device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restri
     }
 }
 
+// ---------------------------------------------------------------------------
+// Version 2: the paper's V2 search (PAPER.md:1@13703-14454 §III.B: "each
+// thread ... is responsible for one character of the uncoded lookahead
+// buffer" and searches the whole window buffer for it; "all the matches are
+// searched ... redundant ones are eliminated" @17800) as the north star's
+// warp-cooperative kernel: for EVERY position p of the chunk the warp
+// evaluates all window offsets at once, lane l taking d = l+1, l+33, l+65,
+// l+97 (l+129, ... for W > 128).  Each offset's run is measured with packed
+// 32-bit compares (XOR of 4 bytes; the first differing byte ends the run, a
+// fully equal word extends it 4 bytes at a time), and the warp's argmax is
+// one __reduce_max_sync over (L << 8) | (255 - (d - 1)): the largest L, ties
+// to the smallest d (reading R7).  L < 3 is a literal (R4).  The result is the
+// same (L, D) table the lazy walk evaluates on demand, so the greedy parse
+// and the bit-pack downstream are shared.  It executes the brute-force
+// compare count of the roofline's compare term.
+__device__ __forceinline__ uint32_t v2_run(const uint32_t *cw, int p, int d, uint32_t p0, int cap) {
+    const int q = p - d;
+    uint32_t x = load4(cw, q) ^ p0;
+    int k = 4;
+    // early out on the first differing byte; equal words extend the run
+    while (!x && k < cap) {
+        x = load4(cw, q + k) ^ load4(cw, p + k);
+        k += 4;
+    }
+    const int L = x ? k - 4 + ((__ffs(x) - 1) >> 3) : k;
+    return (uint32_t)min(L, cap);
+}
+
+__device__ void v2_search_all(const uint32_t *cw, uint16_t *ld, int m, int W, int F, int half, int lane) {
+#pragma unroll 1
+    for (int p = half; p < m; p += kWarpsPerChunk) {
+        const int cap = min(F, m - p);
+        const int dmax = min(W, p);
+        uint32_t best = 0;
+        if (cap >= 3) {
+            const uint32_t p0 = load4(cw, p);  // same word for every lane (broadcast)
+#pragma unroll 4
+            for (int d = lane + 1; d <= dmax; d += 32) {
+                const uint32_t L = v2_run(cw, p, d, p0, cap);
+                const uint32_t key = L >= 3 ? (L << 8) | (uint32_t)(256 - d) : 0u;
+                best = max(best, key);
+            }
+        }
+        best = __reduce_max_sync(kFull, best);
+        if (lane == 0) ld[sk2(p)] = best ? (uint16_t)(((256 - (best & 0xFF)) << 8) | ((best >> 8) - 3)) : kLit;
+    }
+}
+
+// greedy parse over a fully evaluated token table: jump from p to the end of
+// segment [.., s1); returns the exit (first position >= s1 on the path)
+__device__ __forceinline__ int v2_jump(const uint16_t *ld, int p, int s1) {
+#pragma unroll 1
+    while (p < s1) p += tok_len(ld[sk2(p)]);
+    return p;
+}
+
 __device__ __forceinline__ void pair_sync(int id) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(kWalkLanes) : "memory");
 }
 
-template <int MODE, bool SMALLW>
+template <int MODE, bool SMALLW, bool V2>
 __global__ void __launch_bounds__(kChunksPerCta * kWalkLanes, kCtasPerSm)
 chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__restrict__ bucket,
              uint32_t *__restrict__ sizes, void *__restrict__ dbg) {
@@ -298,7 +354,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     // Lane l of warp 0 owns the 128-position build segment [128 l, 128 l + 128)
     // and its own hash table; straight-line: every position is hashed and
     // inserted; the last two positions (no 3-gram) get link 0 after.
-    if (half == 0) {
+    if (!V2 && half == 0) {
         const int b0 = lane * kSeg;
         const int b1 = min(b0 + kSeg, m);
         unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + (SMALLW ? lane : 2 * lane);
@@ -356,12 +412,17 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         }
     }
     pair_sync(bar);  // tab is dead from here on
+    if (V2) {
+        // version 2: (L, D) of every position by the warp-cooperative search
+        v2_search_all(sm.cw, sm.a.u.w.ld, m, W, F, half, lane);
+        pair_sync(bar);
+    }
 
     if (MODE == kModeDumpMatch) {
         // every position, for per-position parity (a2)
         uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
         for (int p = t64; p < m; p += kWalkLanes) {
-            const uint32_t t = eval_pos(sm.cw, link, p, m, W, F);
+            const uint32_t t = V2 ? (uint32_t)sm.a.u.w.ld[sk2(p)] : eval_pos(sm.cw, link, p, m, W, F);
             LD[2 * p] = (uint8_t)(t == kLit ? 0 : (t & 0xFF) + 3);
             LD[2 * p + 1] = (uint8_t)(t == kLit ? 0 : t >> 8);
         }
@@ -373,7 +434,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     const int s1 = min(s0 + kWSeg, m);  // <= s0 for lanes past the chunk end
     uint16_t *ld = sm.a.u.w.ld;
     uint32_t *ucw = sm.a.u.w.ucw;
-    {
+    if (!V2) {
         // zero the memoised tokens (their bytes held the hash tables) and
         // unskew the chunk for the walks' compares
         uint4 *l4 = reinterpret_cast<uint4 *>(ld);
@@ -383,7 +444,12 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     }
     // candidate mask: bit i = position s0 + i (< s1) has a chain link
     uint32_t rc0 = 0, rc1 = 0;
-    if (s0 < s1) {
+    if (V2) {
+        // every position holds its evaluated token
+        const int r = max(s1 - s0, 0);
+        rc0 = r >= 32 ? 0xFFFFFFFFu : ~(0xFFFFFFFFu >> r);
+        rc1 = r <= 32 ? 0u : (r >= 64 ? 0xFFFFFFFFu : ~(0xFFFFFFFFu >> (r - 32)));
+    } else if (s0 < s1) {
         const int so = (s0 >> 7) << 2;  // constant skew inside the segment
         uint32_t h[2] = {0, 0};
 #pragma unroll
@@ -401,7 +467,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         rc1 = __brev(h[1]);
     }
     pair_sync(bar);
-    const int spec_exit = walk_spec(ucw, link, rc0, rc1, ld, m, W, F, s0, s1);
+    const int spec_exit = V2 ? v2_jump(ld, s0, s1) : walk_spec(ucw, link, rc0, rc1, ld, m, W, F, s0, s1);
     int exitp = spec_exit;
     int cur = s0;
     bool first = true;
@@ -425,7 +491,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         pair_sync(bar);  // xf is reused by the next round
         if (!go) break;
         if (chg) {
-            exitp = walk_fix(sm.cw, link, rc0, rc1, ld, m, W, F, s0, s1, entry, spec_exit, first);
+            exitp = V2 ? v2_jump(ld, entry, s1)
+                       : walk_fix(sm.cw, link, rc0, rc1, ld, m, W, F, s0, s1, entry, spec_exit, first);
             first = false;
             cur = entry;
         }
@@ -553,7 +620,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     if (t64 == 0) sizes[c] = (uint32_t)nbytes;
 }
 
-template <int MODE, bool SMALLW>
+template <int MODE, bool SMALLW, bool V2>
 cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *bucket,
                         uint32_t *sizes, void *dbg, cudaStream_t st) {
     const uint64_t C = (n + g.S - 1) / g.S;
@@ -561,13 +628,13 @@ cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *buck
     const size_t smem = sizeof(WarpSmem) * kChunksPerCta;
     static bool attr_set = false;  // benign race: idempotent
     if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(chunk_kernel<MODE, SMALLW>,
+        cudaError_t e = cudaFuncSetAttribute(chunk_kernel<MODE, SMALLW, V2>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         attr_set = true;
     }
     const uint64_t blocks = (C + kChunksPerCta - 1) / kChunksPerCta;
-    chunk_kernel<MODE, SMALLW><<<(unsigned)blocks, kChunksPerCta * kWalkLanes, smem, st>>>(in, n, g, bucket,
+    chunk_kernel<MODE, SMALLW, V2><<<(unsigned)blocks, kChunksPerCta * kWalkLanes, smem, st>>>(in, n, g, bucket,
                                                                                             sizes, dbg);
     count_launch();
     return cudaGetLastError();
@@ -576,8 +643,9 @@ cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *buck
 template <int MODE>
 cudaError_t launch_w(const uint8_t *in, uint64_t n, Geometry g, uint8_t *bucket, uint32_t *sizes,
                      void *dbg, cudaStream_t st) {
-    return g.W <= 128 ? launch_mode<MODE, true>(in, n, g, bucket, sizes, dbg, st)
-                      : launch_mode<MODE, false>(in, n, g, bucket, sizes, dbg, st);
+    if (g.V == 2) return launch_mode<MODE, false, true>(in, n, g, bucket, sizes, dbg, st);
+    return g.W <= 128 ? launch_mode<MODE, true, false>(in, n, g, bucket, sizes, dbg, st)
+                      : launch_mode<MODE, false, false>(in, n, g, bucket, sizes, dbg, st);
 }
 
 }  // namespace
