@@ -409,6 +409,34 @@ def main():
                               "roundtrip_exact": ok}
         del dec
 
+    # NEXT-1 sharded decompression at N > 1: every rank decodes its own chunk
+    # range from its compress_chunks payload + sizes (no exchange needed);
+    # aggregate output GB/s over the max-over-ranks device time
+    if world > 1 and not args.no_decompress:
+        dec = torch.empty(n, dtype=torch.uint8, device=dev)
+        tpay = culzss.compress_chunks(x, payload, sizes)
+        dms = []
+        for it in range(args.warmup + args.steps):
+            flush.fill_(1)
+            torch.cuda.synchronize()
+            ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            ev0.record(stream)
+            culzss.decompress_chunks(payload[:tpay], sizes[:C], n, dec)
+            ev1.record(stream)
+            ev1.synchronize()
+            if it >= args.warmup:
+                dms.append(ev0.elapsed_time(ev1))
+        ok = torch.tensor([1.0 if torch.equal(dec, x) else 0.0], dtype=torch.float64,
+                          device=dev if backend == "nccl" else None)
+        tt = torch.tensor([statistics.mean(dms)], dtype=torch.float64, device=dev if backend == "nccl" else None)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        line["decompress"] = {"value": n_total / (float(tt.item()) / 1000) / 1e9, "unit": "GB/s (output)",
+                              "call_ms_max_over_ranks": float(tt.item()),
+                              "api": "culzss_decompress_chunks (each rank its own chunk range)",
+                              "roundtrip_exact": bool(ok.item() == 1.0)}
+        del dec
+
     if not args.no_e2e:
         hin = torch.from_numpy(x_np).pin_memory()
         hout = torch.empty(culzss.max_compressed_size(n), dtype=torch.uint8).pin_memory()

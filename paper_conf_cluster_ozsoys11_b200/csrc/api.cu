@@ -594,6 +594,44 @@ culzss_status culzss_decompressed_size(const void *in, size_t in_n, size_t *n,
     return s == CULZSS_ERR_UNSUPPORTED ? CULZSS_OK : s;
 }
 
+// Decode C chunks (n output bytes) from `payload` (pay_len bytes) with the
+// u32 size table at `table_src` (device, any alignment: copied to an aligned
+// workspace).  Scan of the sizes, walk + decode kernels, one sync for the
+// device error word.
+static culzss_status decompress_core(const uint8_t *payload, uint64_t pay_len, const void *table_src, uint64_t C,
+                                     uint64_t n, const Geometry &g, uint8_t *out, cudaStream_t st) {
+    // workspace: aligned copy of the table | offsets | scan ws | total | err
+    const uint64_t tab_off = 0;
+    const uint64_t offs_off = (C * 4 + 255) / 256 * 256;
+    const uint64_t ws_off = offs_off + (C * 8 + 255) / 256 * 256;
+    const uint64_t tot_off = ws_off + (scan_workspace_words(C) * 8 + 255) / 256 * 256;
+    const uint64_t tb_off = tot_off + 256;
+    Workspace ws(st);
+    CK(ws.alloc(tb_off + decode_scratch_bytes(C)));
+    uint8_t *base = static_cast<uint8_t *>(ws.p);
+    uint32_t *sizes = reinterpret_cast<uint32_t *>(base + tab_off);
+    uint64_t *offsets = reinterpret_cast<uint64_t *>(base + offs_off);
+    uint64_t *scanws = reinterpret_cast<uint64_t *>(base + ws_off);
+    uint64_t *total = reinterpret_cast<uint64_t *>(base + tot_off);
+    uint32_t *err = reinterpret_cast<uint32_t *>(base + tot_off + 8);
+    CK(cudaMemcpyAsync(sizes, table_src, C * 4, cudaMemcpyDeviceToDevice, st));
+    CK(cudaMemsetAsync(err, 0, 4, st));
+    CK(launch_scan(sizes, C, offsets, total, scanws, st));
+    uint64_t *hw = host_word();
+    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
+    // the walk kernel checks the table against the payload length (no sync here)
+    t_prof.reset();
+    t_prof.rec(1, st);
+    CK(launch_decode(payload, pay_len, sizes, offsets, C, n, g, out, err, reinterpret_cast<uint32_t *>(base + tb_off),
+                     st));
+    t_prof.rec(2, st);
+    CK(cudaMemcpyAsync(hw, err, 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (t_profiling) t_times.decode = t_prof.between(1, 2);
+    if (reinterpret_cast<uint32_t *>(hw)[0]) return CULZSS_ERR_CORRUPT;
+    return CULZSS_OK;
+}
+
 culzss_status culzss_decompress(const void *in, size_t in_n, void *out, size_t *out_n,
                                 const culzss_params *, culzss_stream_t stream) {
     lib_init();
@@ -615,38 +653,27 @@ culzss_status culzss_decompress(const void *in, size_t in_n, void *out, size_t *
         return CULZSS_OK;
     }
     if (!is_device_ptr(out) || overlap(in, in_n, out, n)) return CULZSS_ERR_INVALID_ARG;
-    // workspace: aligned copy of the table | offsets | scan ws | total | err
-    const uint64_t tab_off = 0;
-    const uint64_t offs_off = (C * 4 + 255) / 256 * 256;
-    const uint64_t ws_off = offs_off + (C * 8 + 255) / 256 * 256;
-    const uint64_t tot_off = ws_off + (scan_workspace_words(C) * 8 + 255) / 256 * 256;
-    const uint64_t tb_off = tot_off + 256;
-    Workspace ws(st);
-    CK(ws.alloc(tb_off + decode_scratch_bytes(C)));
-    uint8_t *base = static_cast<uint8_t *>(ws.p);
-    uint32_t *sizes = reinterpret_cast<uint32_t *>(base + tab_off);
-    uint64_t *offsets = reinterpret_cast<uint64_t *>(base + offs_off);
-    uint64_t *scanws = reinterpret_cast<uint64_t *>(base + ws_off);
-    uint64_t *total = reinterpret_cast<uint64_t *>(base + tot_off);
-    uint32_t *err = reinterpret_cast<uint32_t *>(base + tot_off + 8);
     const uint8_t *src = static_cast<const uint8_t *>(in);
-    CK(cudaMemcpyAsync(sizes, src + 32, C * 4, cudaMemcpyDeviceToDevice, st));
-    CK(cudaMemsetAsync(err, 0, 4, st));
-    CK(launch_scan(sizes, C, offsets, total, scanws, st));
-    uint64_t *hw = host_word();
-    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
-    // the walk kernel checks the table against the payload length (no sync here)
-    t_prof.reset();
-    t_prof.rec(1, st);
-    CK(launch_decode(src + 32 + 4 * C, in_n - 32 - 4 * C, sizes, offsets, C, n, g, static_cast<uint8_t *>(out),
-                     err, reinterpret_cast<uint32_t *>(base + tb_off), st));
-    t_prof.rec(2, st);
-    CK(cudaMemcpyAsync(hw, err, 4, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    if (t_profiling) t_times.decode = t_prof.between(1, 2);
-    if (reinterpret_cast<uint32_t *>(hw)[0]) return CULZSS_ERR_CORRUPT;
-    *out_n = (size_t)n;
-    return CULZSS_OK;
+    s = decompress_core(src + 32 + 4 * C, in_n - 32 - 4 * C, src + 32, C, n, g, static_cast<uint8_t *>(out), st);
+    if (s == CULZSS_OK) *out_n = (size_t)n;
+    return s;
+}
+
+culzss_status culzss_decompress_chunks(const void *payload, size_t payload_n, const uint32_t *chunk_sizes,
+                                       size_t slice_n, void *out, const culzss_params *p,
+                                       culzss_stream_t stream) {
+    lib_init();
+    if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
+    Geometry g;
+    culzss_status s = check_params(p, &g);
+    if (s != CULZSS_OK) return s;
+    if (slice_n == 0) return payload_n == 0 ? CULZSS_OK : CULZSS_ERR_CORRUPT;
+    const uint64_t C = n_chunks(slice_n, g.S);
+    if (!is_device_ptr(payload) || !is_device_ptr(chunk_sizes) || !is_device_ptr(out) ||
+        overlap(payload, payload_n, out, slice_n) || overlap(chunk_sizes, 4 * C, out, slice_n))
+        return CULZSS_ERR_INVALID_ARG;
+    return decompress_core(static_cast<const uint8_t *>(payload), payload_n, chunk_sizes, C, slice_n, g,
+                           static_cast<uint8_t *>(out), (cudaStream_t)stream);
 }
 
 static culzss_status debug_entry(int mode, const void *in, size_t n, void *dst,

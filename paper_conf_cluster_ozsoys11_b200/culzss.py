@@ -68,6 +68,7 @@ def _lib():
         L.culzss_decompressed_size.argtypes = [vp, sz, szp, vp]
         L.culzss_decompress.argtypes = [vp, sz, vp, szp, pp, vp]
         L.culzss_compress_chunks.argtypes = [vp, sz, vp, szp, vp, pp, vp]
+        L.culzss_decompress_chunks.argtypes = [vp, sz, vp, sz, vp, pp, vp]
         L.culzss_write_header.argtypes = [vp, sz, pp, vp]
         L.culzss_match_search.argtypes = [vp, sz, vp, pp, vp]
         L.culzss_parse_tokens.argtypes = [vp, sz, vp, pp, vp]
@@ -218,6 +219,32 @@ def compress_chunks(x_slice, payload, chunk_sizes, params: Optional[Params] = No
                                        _stream(stream))
     _check(st, "culzss_compress_chunks")
     return pn.value
+
+
+def decompress_chunks_status(payload, chunk_sizes, slice_n: int, out=None, params: Optional[Params] = None,
+                             stream=None) -> Tuple[int, object]:
+    """Sharded decompression (inverse of compress_chunks): decode the
+    ceil(slice_n/S) chunks of `payload` (CUDA uint8) sized by `chunk_sizes`
+    (CUDA int32, u32 bit pattern) into `out` (CUDA uint8, slice_n bytes)."""
+    import torch
+    _dev_u8(payload)
+    if not (chunk_sizes.is_cuda and chunk_sizes.dtype == torch.int32):
+        raise TypeError("chunk_sizes must be a CUDA int32 tensor (u32 bit pattern)")
+    if out is None:
+        out = torch.empty(max(slice_n, 1), dtype=torch.uint8, device=payload.device)
+    _dev_u8(out)
+    if out.numel() < slice_n:
+        raise ValueError("out is smaller than slice_n")
+    st = _lib().culzss_decompress_chunks(ctypes.c_void_p(payload.data_ptr()), payload.numel(),
+                                         ctypes.c_void_p(chunk_sizes.data_ptr()), slice_n,
+                                         ctypes.c_void_p(out.data_ptr()), _params(params), _stream(stream))
+    return st, (out[:slice_n] if st == OK else None)
+
+
+def decompress_chunks(payload, chunk_sizes, slice_n: int, out=None, params: Optional[Params] = None, stream=None):
+    st, o = decompress_chunks_status(payload, chunk_sizes, slice_n, out, params, stream)
+    _check(st, "culzss_decompress_chunks")
+    return o
 
 
 def write_header(out, n_total: int, params: Optional[Params] = None, stream=None) -> None:

@@ -76,6 +76,28 @@ def placements(totals: Sequence[int], n: int, S: int) -> List[RankPlacement]:
     return out
 
 
+def stream_views(sizes: Sequence[int], n: int, S: int, world: int) -> List[RankPlacement]:
+    """Sharded decompression of an existing stream:
+    from its u32 size table (host copy, C entries), rank r decodes chunks
+    [c0, c1) = chunk_range(r, world, C) -- table slice at 32 + 4 c0, payload
+    at 32 + 4 C + sum(sizes[:c0]) of length sum(sizes[c0:c1]) -- into output
+    bytes [c0 S, min(c1 S, n)).  No exchange is needed: the table is in the
+    stream."""
+    C = n_chunks(n, S)
+    if len(sizes) != C:
+        raise ValueError("size table length != ceil(n / S)")
+    base = HEADER_BYTES + 4 * C
+    prefix = [0]
+    for v in sizes:
+        prefix.append(prefix[-1] + int(v))
+    out = []
+    for r in range(world):
+        c0, c1 = chunk_range(r, world, C)
+        out.append(RankPlacement(r, c0, c1, HEADER_BYTES + 4 * c0, base + prefix[c0],
+                                 prefix[c1] - prefix[c0], base + prefix[-1]))
+    return out
+
+
 def exchange_totals(my_total: int, group=None, device=None) -> List[int]:
     """The one collective: all-gather of int64 per-rank payload totals."""
     import torch

@@ -80,3 +80,60 @@ def test_placements_closed_form():
     assert pl[3].table_offset == 32 + 4 * 8
     assert all(p.stream_bytes == 32 + 4 * C + 363 for p in pl)
     assert sharding.header(n)[:4] == b"CLZS" and len(sharding.header(n)) == 32
+
+
+def _dec_worker(rank, world, port, kind, n, S, out_q):
+    """Sharded decompression on CPU: every rank decodes its own chunk range of
+    the stream (a header + its table slice + its payload slice is itself a
+    valid stream of the slice), rank 0 gathers the slices."""
+    import torch.distributed as dist
+    import oracle as O
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        x = datagen.generate(kind, n, seed=23)
+        stream = O.compress(x, S=S)
+        C = sharding.n_chunks(n, S)
+        sizes = np.frombuffer(stream, "<u4", count=C, offset=32).tolist()
+        v = sharding.stream_views(sizes, n, S, world)[rank]
+        b0, b1 = sharding.byte_range(rank, world, n, S)
+        mini = (sharding.header(b1 - b0, S) + stream[v.table_offset:v.table_offset + 4 * (v.c1 - v.c0)]
+                + stream[v.payload_offset:v.payload_offset + v.payload_bytes])
+        part = O.decompress(mini)
+        objs = [None] * world if rank == 0 else None
+        dist.gather_object((rank, part), objs, dst=0)
+        if rank == 0:
+            out_q.put(b"".join(p for _, p in sorted(objs)))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,kind,n,S", [(2, "csource", 37 * 4096 + 1111, 4096),
+                                            (3, "tarmix", 5000, 1000),
+                                            (4, "runs20", 2 * 4096 + 7, 4096)])
+def test_sharded_decompress_gloo(world, kind, n, S):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_dec_worker, args=(r, world, port, kind, n, S, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert out == datagen.generate(kind, n, seed=23).tobytes()
+
+
+def test_stream_views_closed_form():
+    n, S = 10 * 4096 + 7, 4096
+    sizes = [10, 20, 30, 40, 50, 60, 70, 80, 90, 100, 5]
+    v = sharding.stream_views(sizes, n, S, 4)
+    C = 11
+    assert [(p.c0, p.c1) for p in v] == [(0, 2), (2, 5), (5, 8), (8, 11)]
+    assert [p.payload_offset for p in v] == [32 + 4 * C + o for o in (0, 30, 150, 360)]
+    assert [p.payload_bytes for p in v] == [30, 120, 210, 195]
+    assert all(p.stream_bytes == 32 + 4 * C + sum(sizes) for p in v)
+    with pytest.raises(ValueError):
+        sharding.stream_views(sizes[:-1], n, S, 2)
