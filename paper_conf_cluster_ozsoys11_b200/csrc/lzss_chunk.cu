@@ -154,7 +154,7 @@ __device__ uint32_t eval_pos(const uint32_t *cw, const uint8_t *link, int p, int
 __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const uint8_t *__restrict__ link,
                                          uint32_t rc0, uint32_t rc1, uint16_t *__restrict__ ld, int m, int W,
                                          int F, int s0,
-                                         int s1) {
+                                         int s1, bool &anym) {
     // token starts stay inside the lane's segment, which never crosses a
     // 128-position skew boundary: p-indexed arrays use a constant offset
     const int so = (s0 >> 7) << 2;
@@ -162,6 +162,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
     uint16_t *lds = ld + (so >> 1);
     int p = next_cand(rc0, rc1, s0, s0, s1);
     bool active = p < s1;
+    uint32_t nm = 0;  // matches found on the path
     int d = 0, cap = 0;
     if (active) {
         d = lks[p];
@@ -177,7 +178,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
             const int lq = link[sk(q)];  // next chain member, loaded with the compare words
             const Be8 vq = load8(u, q + off), vp = load8(u, p + off);
             const uint32_t xh = vq.hi ^ vp.hi, xl = vq.lo ^ vp.lo;
-            const int fb = xh ? __clz(xh) >> 3 : 4 + (__clz(xl) >> 3);  // equal leading bytes (<= 8)
+            const int fb = __clzll(((uint64_t)xh << 32) | xl) >> 3;  // equal leading bytes (<= 8), branch-free
             const bool cand_done = qr ? xh != 0 : (fb < 8 || k + 8 >= cap);
             const int L = min(k + fb, cap);
             const bool upd = !qr && cand_done && L > bestL;
@@ -196,6 +197,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
             }
             if (tok_done) {
                 lds[p] = (uint16_t)(bestD ? (bestD << 8) | (bestL - 3) : kLit);
+                nm |= bestD;
                 p = next_cand(rc0, rc1, p + (bestD ? bestL : 1), s0, s1);
                 active = p < s1;
                 if (active) {
@@ -209,6 +211,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
             }
         }
     }
+    anym = nm != 0;
     return p;
 }
 
@@ -467,7 +470,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         rc1 = __brev(h[1]);
     }
     pair_sync(bar);
-    const int spec_exit = V2 ? v2_jump(ld, s0, s1) : walk_spec(ucw, link, rc0, rc1, ld, m, W, F, s0, s1);
+    bool anym = true;  // the speculative path holds a match (V2: not tracked)
+    const int spec_exit = V2 ? v2_jump(ld, s0, s1) : walk_spec(ucw, link, rc0, rc1, ld, m, W, F, s0, s1, anym);
     int exitp = spec_exit;
     int cur = s0;
     bool first = true;
@@ -536,6 +540,29 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         const uint32_t *ldw = reinterpret_cast<const uint32_t *>(ld + (so >> 1) + s0);  // 2 tokens / word
         const uint32_t *cbw = reinterpret_cast<const uint32_t *>(cb + so + s0);         // 4 bytes / word
         const int ng = (s1 - s0 + 3) >> 2;
+        if (__all_sync(kFull, !anym && cur == s0 && s1 - s0 == kWSeg)) {
+            // every lane of the warp walks its whole segment from its start
+            // and found no match: 64 literals each (incompressible data),
+            // emitted branch-free in 18-bit pairs (bit positions static)
+#pragma unroll
+            for (int i = 0; i < kWSeg / 4; i++) {
+                const uint32_t bytes = cbw[i];
+                const uint32_t v0 = ((bytes & 0xFFu) << 9) | ((bytes >> 8) & 0xFFu);
+                const uint32_t v1 = (((bytes >> 16) & 0xFFu) << 9) | (bytes >> 24);
+                acc = (acc << 18) | v0;
+                nacc += 18;
+                if (nacc >= 32) {
+                    nacc -= 32;
+                    stage[nw++] = (uint32_t)(acc >> nacc);
+                }
+                acc = (acc << 18) | v1;
+                nacc += 18;
+                if (nacc >= 32) {
+                    nacc -= 32;
+                    stage[nw++] = (uint32_t)(acc >> nacc);
+                }
+            }
+        } else
 #pragma unroll 1
         for (int i = max(0, (cov - s0) >> 2); i < ng; i = max(i + 1, (cov - s0) >> 2)) {
             // groups wholly inside a match are skipped
