@@ -193,7 +193,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
                 tok_done = l2 == 0 || nd > W;
                 d = nd;
                 k = 0;
-                qr = bestL >= 3;
+                qr = bestL >= 8;  // below 8 the first 8-byte LCP step decides as cheaply
             }
             if (tok_done) {
                 lds[p] = (uint16_t)(bestD ? (bestD << 8) | (bestL - 3) : kLit);
