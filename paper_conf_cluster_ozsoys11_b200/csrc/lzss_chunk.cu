@@ -143,8 +143,10 @@ __device__ uint32_t eval_pos(const uint32_t *cw, const uint8_t *link, int p, int
 // state machine: every iteration of every active lane does exactly one
 // 8-byte compare of its current candidate d at offset `off` (on the unskewed
 // chunk copy u) and then updates its state with selects:
-//   * a candidate first gets a 4-byte reject test at offset bestL-3 (it can
-//     only win if bytes [0, bestL] match), then its LCP 8 bytes per iteration;
+//   * once bestL >= 8 a candidate first gets an 8-byte reject test of bytes
+//     [bestL-7, bestL] (it can only win if bytes [0, bestL] match); then (or
+//     directly, below 8, where the first LCP step decides as cheaply) its
+//     LCP 8 bytes per iteration;
 //   * a finished candidate moves to the next one on the hash chain
 //     (d += link[p-d]) or finishes the token;
 //   * a finished token is memoised in ld[] and p jumps over candidate-free
@@ -174,18 +176,18 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
     while (__any_sync(kFull, active)) {
         if (active) {
             const int q = p - d;
-            const int off = qr ? bestL - 3 : k;
+            const int off = qr ? bestL - 7 : k;
             const int lq = link[sk(q)];  // next chain member, loaded with the compare words
             const Be8 vq = load8(u, q + off), vp = load8(u, p + off);
             const uint32_t xh = vq.hi ^ vp.hi, xl = vq.lo ^ vp.lo;
             const int fb = __clzll(((uint64_t)xh << 32) | xl) >> 3;  // equal leading bytes (<= 8), branch-free
-            const bool cand_done = qr ? xh != 0 : (fb < 8 || k + 8 >= cap);
+            const bool cand_done = fb < 8 || (!qr && k + 8 >= cap);
             const int L = min(k + fb, cap);
             const bool upd = !qr && cand_done && L > bestL;
             bestL = upd ? L : bestL;
             bestD = upd ? d : bestD;
             k = qr ? 0 : k + 8;
-            qr = qr && xh != 0;
+            qr = qr && fb < 8;
             bool tok_done = false;
             if (cand_done) {
                 const int l2 = bestL == cap ? 0 : lq;
@@ -193,7 +195,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
                 tok_done = l2 == 0 || nd > W;
                 d = nd;
                 k = 0;
-                qr = bestL >= 8;  // below 8 the first 8-byte LCP step decides as cheaply
+                qr = bestL >= 8;
             }
             if (tok_done) {
                 lds[p] = (uint16_t)(bestD ? (bestD << 8) | (bestL - 3) : kLit);
