@@ -536,12 +536,22 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         // wrote it, and is 0 for candidate-free positions (literals).  Each
         // position emits 0, 9 or 17 bits.
         uint64_t acc = 0;
-        int nacc = 0, nw = 0;
+        int nacc = 0;
+        uint32_t *sp = stage;  // next staging word
         int cov = cur;  // positions < cov are covered (by the previous lane or a match)
         const int so = (s0 >> 7) << 2;
         const uint32_t *ldw = reinterpret_cast<const uint32_t *>(ld + (so >> 1) + s0);  // 2 tokens / word
         const uint32_t *cbw = reinterpret_cast<const uint32_t *>(cb + so + s0);         // 4 bytes / word
         const int ng = (s1 - s0 + 3) >> 2;
+        // append pn (<= 26) bits; acc keeps < 32 pending bits between calls
+        auto put = [&](uint32_t pv, int pn) {
+            acc = (acc << pn) | pv;
+            nacc += pn;
+            if (nacc >= 32) {
+                nacc -= 32;
+                *sp++ = (uint32_t)(acc >> nacc);
+            }
+        };
         if (__all_sync(kFull, !anym && cur == s0 && s1 - s0 == kWSeg)) {
             // every lane of the warp walks its whole segment from its start
             // and found no match: 64 literals each (incompressible data),
@@ -549,27 +559,19 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
 #pragma unroll
             for (int i = 0; i < kWSeg / 4; i++) {
                 const uint32_t bytes = cbw[i];
-                const uint32_t v0 = ((bytes & 0xFFu) << 9) | ((bytes >> 8) & 0xFFu);
-                const uint32_t v1 = (((bytes >> 16) & 0xFFu) << 9) | (bytes >> 24);
-                acc = (acc << 18) | v0;
-                nacc += 18;
-                if (nacc >= 32) {
-                    nacc -= 32;
-                    stage[nw++] = (uint32_t)(acc >> nacc);
-                }
-                acc = (acc << 18) | v1;
-                nacc += 18;
-                if (nacc >= 32) {
-                    nacc -= 32;
-                    stage[nw++] = (uint32_t)(acc >> nacc);
-                }
+                put(((bytes & 0xFFu) << 9) | ((bytes >> 8) & 0xFFu), 18);
+                put((((bytes >> 16) & 0xFFu) << 9) | (bytes >> 24), 18);
             }
         } else
 #pragma unroll 1
         for (int i = max(0, (cov - s0) >> 2); i < ng; i = max(i + 1, (cov - s0) >> 2)) {
-            // groups wholly inside a match are skipped
+            // groups wholly inside a match are skipped.  Positions are
+            // combined in pairs in 32 bits first: a pair is at most a literal
+            // and a match (26 bits), since a match covers the next position.
             const uint32_t bytes = cbw[i];
             const uint32_t t01 = ldw[2 * i], t23 = ldw[2 * i + 1];
+            uint32_t pv = 0;
+            int pn = 0;
 #pragma unroll
             for (int j = 0; j < 4; j++) {
                 const int p = s0 + 4 * i + j;
@@ -577,18 +579,20 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                 const bool on = p >= cov && p < s1;
                 const bool mt = on && t >= 0x100;
                 const int nb = mt ? 17 : (on ? 9 : 0);
-                const uint32_t val = mt ? t + (0x10000u - 0x100u) : (bytes >> (8 * j)) & 0xFFu;  // 1|D-1|L-3
+                const uint32_t val = mt ? t + (0x10000u - 0x100u) : (on ? (bytes >> (8 * j)) & 0xFFu : 0u);  // 1|D-1|L-3
                 cov = mt ? p + (int)(t & 0xFF) + 3 : cov;
-                acc = (acc << nb) | (nb ? val : 0u);
-                nacc += nb;
-                if (nacc >= 32) {
-                    nacc -= 32;
-                    stage[nw++] = (uint32_t)(acc >> nacc);
+                pv = (pv << nb) | val;
+                pn += nb;
+                if (j & 1) {
+                    put(pv, pn);
+                    pv = 0;
+                    pn = 0;
                 }
             }
         }
+        const int nw = (int)(sp - stage);
         nbits = 32 * nw + nacc;
-        if (nacc > 0) stage[nw] = (uint32_t)(acc << (32 - nacc));
+        if (nacc > 0) *sp = (uint32_t)(acc << (32 - nacc));
     }
     // exclusive scan of bit counts over the 64 walk lanes
     int incl = nbits;
