@@ -378,6 +378,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                 }
             }
             // own segment: links
+            const uint32_t w4 = (uint32_t)min(W, 255) * 0x01010101u;
 #pragma unroll 1
             for (int wi = 0; wi < 4; wi++) {
                 const int pb = b0 + 32 * wi;
@@ -387,22 +388,30 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                         const int p = pb + 4 * i;
                         const uint32_t w0 = sm.cw[sk(p) >> 2], w1 = sm.cw[(sk(p) >> 2) + 1];
                         uint32_t lw = 0;
+                        if (SMALLW) {
+                            // entries hold position mod 256: every live entry is
+                            // within 256 of p, the empty value maps to 0 or > 128.
+                            // Entries are read and replaced in position order
+                            // (a repeated hash in the group sees its predecessor),
+                            // then the four distances are formed bytewise.
+                            uint32_t E = 0;
 #pragma unroll
-                        for (int j = 0; j < 4; j++) {
-                            const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
-                            uint32_t dist;
-                            if (SMALLW) {
-                                // entries hold position mod 256: every live entry is
-                                // within 256 of p, the empty value maps to 0 or > 128
-                                uint8_t *e = tabl + hash_off9(key);
-                                dist = (uint32_t)(p + j - *e) & 0xFFu;
+                            for (int j = 0; j < 4; j++) {
+                                uint8_t *e = tabl + hash_off9(__funnelshift_r(w0, w1, 8 * j));
+                                E |= (uint32_t)*e << (8 * j);
                                 *e = (uint8_t)(p + j);
-                            } else {
-                                uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(key));
-                                dist = (uint32_t)(p + j + kTabBias) - *e;
-                                *e = (uint16_t)(p + j + kTabBias);
                             }
-                            lw |= (dist <= (uint32_t)W ? dist : 0u) << (8 * j);
+                            const uint32_t D = __vsub4(__vadd4(((uint32_t)p & 0xFFu) * 0x01010101u, 0x03020100u), E);
+                            lw = D & __vcmpleu4(D, w4);  // distance, or 0 past the window
+                        } else {
+#pragma unroll
+                            for (int j = 0; j < 4; j++) {
+                                const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
+                                uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(key));
+                                const uint32_t dist = (uint32_t)(p + j + kTabBias) - *e;
+                                *e = (uint16_t)(p + j + kTabBias);
+                                lw |= (dist <= (uint32_t)W ? dist : 0u) << (8 * j);
+                            }
                         }
                         *reinterpret_cast<uint32_t *>(link + sk(p)) = lw;
                     }
