@@ -103,8 +103,10 @@ __device__ __forceinline__ bool is_cand(uint32_t rc0, uint32_t rc1, int o) {
 // little-endian word whose low 3 bytes are the 3-gram: hash h = top 8 bits of
 // (w << 8) * K (== w * (K << 8)); entry [h][lane] lives at byte 64 h + 2 lane
 __device__ __forceinline__ uint32_t hash_off(uint32_t w) { return ((w * kHashMul) >> 18) & 0x3FC0u; }
-// W <= 128 variant: 9-bit hash, u8 entries [h][lane] at byte 32 h + lane
-__device__ __forceinline__ uint32_t hash_off9(uint32_t w) { return ((w * kHashMul) >> 18) & 0x3FE0u; }
+// W <= 128 variant: 9-bit hash h of the same product, u8 entries [lane][h]
+// at byte 512 lane + h (one add per address; lanes' buckets are random, so
+// the bank spread is the same as the interleaved layout's)
+__device__ __forceinline__ uint32_t hash9(uint32_t w) { return (w * kHashMul) >> 23; }
 
 __device__ __forceinline__ int tok_len(uint32_t t) { return t >= 0x100 ? (int)(t & 0xFF) + 3 : 1; }
 
@@ -328,10 +330,12 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         for (int i = t64; i < (int)(sizeof(sm.cw) / 16); i += kWalkLanes) z4[i] = z;
         uint4 *t4 = reinterpret_cast<uint4 *>(sm.a.u.tab);
         // u8 tables: empty = (s0 - 129) mod 256 = 0x7F (even lanes) / 0xFF (odd)
-        const uint32_t e = SMALLW ? 0xFF7FFF7Fu : 0u;
-        const uint4 te = make_uint4(e, e, e, e);
 #pragma unroll 4
-        for (int i = t64; i < (int)(sizeof(sm.a.u.tab) / 16); i += kWalkLanes) t4[i] = te;
+        for (int i = t64; i < (int)(sizeof(sm.a.u.tab) / 16); i += kWalkLanes) {
+            // u8 tables: lane (i >> 5)'s 512 bytes hold its empty value
+            const uint32_t e = SMALLW ? ((i >> 5) & 1 ? 0xFFFFFFFFu : 0x7F7F7F7Fu) : 0u;
+            t4[i] = make_uint4(e, e, e, e);
+        }
     }
     pair_sync(bar);
     if ((reinterpret_cast<uintptr_t>(src) & 15) == 0) {
@@ -362,7 +366,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     if (!V2 && half == 0) {
         const int b0 = lane * kSeg;
         const int b1 = min(b0 + kSeg, m);
-        unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + (SMALLW ? lane : 2 * lane);
+        unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + (SMALLW ? 512 * lane : 2 * lane);
         if (b0 < m) {
             // the W positions before the segment (pre-insert, no links)
 #pragma unroll 1
@@ -372,7 +376,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                 for (int j = 0; j < 4; j++) {
                     const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
                     if (SMALLW)
-                        tabl[hash_off9(key)] = (uint8_t)(q + j);
+                        tabl[hash9(key)] = (uint8_t)(q + j);
                     else
                         *reinterpret_cast<uint16_t *>(tabl + hash_off(key)) = (uint16_t)(q + j + kTabBias);
                 }
@@ -397,7 +401,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                             uint32_t E = 0;
 #pragma unroll
                             for (int j = 0; j < 4; j++) {
-                                uint8_t *e = tabl + hash_off9(__funnelshift_r(w0, w1, 8 * j));
+                                uint8_t *e = tabl + hash9(__funnelshift_r(w0, w1, 8 * j));
                                 E |= (uint32_t)*e << (8 * j);
                                 *e = (uint8_t)(p + j);
                             }
