@@ -82,22 +82,14 @@ __device__ __forceinline__ Be8 load8(const uint32_t *__restrict__ u, int x) {
 }
 
 // first candidate position >= p of the lane's segment [s0, s1), or s1 (p if
-// p >= s1 already).  rc0 / rc1: candidate bits of positions s0..s0+31 /
-// s0+32..s0+63, position s0+i at bit 31-i (reversed: next = count of
-// leading zeros)
-__device__ __forceinline__ int next_cand(uint32_t rc0, uint32_t rc1, int p, int s0, int s1) {
+// p >= s1 already).  cm: candidate bits of positions s0..s0+63, position
+// s0+i at bit 63-i (reversed: next = count of leading zeros)
+__device__ __forceinline__ int next_cand(uint64_t cm, int p, int s0, int s1) {
     if (p >= s1) return p;
-    const int o = p - s0;  // < 64
-    const int sh = o & 31;
-    const uint32_t r0 = rc0 << sh;
-    const int n0 = r0 ? o + __clz(r0) : 32 + __clz(rc1);
-    const int n1 = o + __clz(rc1 << sh);  // clz(0) = 32: past the segment
-    return min(s0 + (o < 32 ? n0 : n1), s1);
+    return min(p + __clzll(cm << (p - s0)), s1);  // clz(0) = 64: past the segment
 }
 
-__device__ __forceinline__ bool is_cand(uint32_t rc0, uint32_t rc1, int o) {
-    return ((o < 32 ? rc0 : rc1) << (o & 31)) >> 31;
-}
+__device__ __forceinline__ bool is_cand(uint64_t cm, int o) { return (cm << o) >> 63; }
 
 // byte offset (into the per-lane-interleaved table) of the 3-gram hash of a
 // little-endian word whose low 3 bytes are the 3-gram: hash h = top 8 bits of
@@ -156,7 +148,7 @@ __device__ uint32_t eval_pos(const uint32_t *cw, const uint8_t *link, int p, int
 //     first candidate is loaded in the same iteration.
 // Returns the exit (first position >= s1 the greedy path reaches).
 __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const uint8_t *__restrict__ link,
-                                         uint32_t rc0, uint32_t rc1, uint16_t *__restrict__ ld, int m, int W,
+                                         uint64_t cm, uint16_t *__restrict__ ld, int m, int W,
                                          int F, int s0,
                                          int s1, bool &anym) {
     // token starts stay inside the lane's segment, which never crosses a
@@ -164,7 +156,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
     const int so = (s0 >> 7) << 2;
     const uint8_t *lks = link + so;
     uint16_t *lds = ld + (so >> 1);
-    int p = next_cand(rc0, rc1, s0, s0, s1);
+    int p = next_cand(cm, s0, s0, s1);
     bool active = p < s1;
     uint32_t nm = 0;  // matches found on the path
     int d = 0, cap = 0;
@@ -202,7 +194,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
             if (tok_done) {
                 lds[p] = (uint16_t)(bestD ? (bestD << 8) | (bestL - 3) : kLit);
                 nm |= bestD;
-                p = next_cand(rc0, rc1, p + (bestD ? bestL : 1), s0, s1);
+                p = next_cand(cm, p + (bestD ? bestL : 1), s0, s1);
                 active = p < s1;
                 if (active) {
                     d = lks[p];
@@ -225,12 +217,12 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
 // there is the same.  A later re-walk of the same lane (rare: its entry moved
 // twice) cannot tell which earlier walk a memoised start belongs to and walks
 // to the segment end, reusing memoised tokens.
-__device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link, uint32_t rc0, uint32_t rc1,
+__device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link, uint64_t cm,
                         uint16_t *__restrict__ ld, int m, int W, int F, int s0, int s1, int entry,
                         int spec_exit, bool first) {
     int p = entry;
     while (true) {
-        p = next_cand(rc0, rc1, p, s0, s1);
+        p = next_cand(cm, p, s0, s1);
         if (p >= s1) return p;
         uint32_t t = ld[sk2(p)];
         if (t && first) return spec_exit;
@@ -486,7 +478,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     }
     pair_sync(bar);
     bool anym = true;  // the speculative path holds a match (V2: not tracked)
-    const int spec_exit = V2 ? v2_jump(ld, s0, s1) : walk_spec(ucw, link, rc0, rc1, ld, m, W, F, s0, s1, anym);
+    const uint64_t cm = ((uint64_t)rc0 << 32) | rc1;
+    const int spec_exit = V2 ? v2_jump(ld, s0, s1) : walk_spec(ucw, link, cm, ld, m, W, F, s0, s1, anym);
     int exitp = spec_exit;
     int cur = s0;
     bool first = true;
@@ -511,7 +504,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         if (!go) break;
         if (chg) {
             exitp = V2 ? v2_jump(ld, entry, s1)
-                       : walk_fix(sm.cw, link, rc0, rc1, ld, m, W, F, s0, s1, entry, spec_exit, first);
+                       : walk_fix(sm.cw, link, cm, ld, m, W, F, s0, s1, entry, spec_exit, first);
             first = false;
             cur = entry;
         }
@@ -522,7 +515,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         for (int p = s0; p < s1; p++) tok[p] = 0;
         int p = cur;
         while (p < s1) {
-            if (!is_cand(rc0, rc1, p - s0)) {
+            if (!is_cand(cm, p - s0)) {
                 tok[p] = 1;
                 p++;
             } else {
