@@ -484,24 +484,27 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     int cur = s0;
     bool first = true;
     volatile uint32_t *xf = sm.a.u.w.xfer;
+    // two barriers per round: exits and "changed" flags use slots alternating
+    // with the round's parity, so a slot is rewritten only two rounds later,
+    // after every read of it
+    int par = 0;
 #pragma unroll 1
     while (true) {
         // entry of walk lane t64 = exit of lane t64 - 1 (warp 1 lane 0 reads
         // warp 0 lane 31 through shared memory)
         int entry = __shfl_up_sync(kFull, exitp, 1);
-        if (lane == 31) xf[half] = (uint32_t)exitp;
+        if (lane == 31) xf[2 * par + half] = (uint32_t)exitp;
         pair_sync(bar);
-        if (lane == 0) entry = half ? (int)xf[half - 1] : 0;
+        if (lane == 0) entry = half ? (int)xf[2 * par + half - 1] : 0;
         const bool chg = entry != cur;
         const bool any = __any_sync(kFull, chg);
-        pair_sync(bar);  // all reads of xf done
-        if (lane == 0) xf[half] = any;
+        if (lane == 0) xf[4 + 2 * par + half] = any;
         pair_sync(bar);
         bool go = false;
 #pragma unroll
-        for (int k = 0; k < kWarpsPerChunk; k++) go |= xf[k] != 0;
-        pair_sync(bar);  // xf is reused by the next round
+        for (int k = 0; k < kWarpsPerChunk; k++) go |= xf[4 + 2 * par + k] != 0;
         if (!go) break;
+        par ^= 1;
         if (chg) {
             exitp = V2 ? v2_jump(ld, entry, s1)
                        : walk_fix(sm.cw, link, cm, ld, m, W, F, s0, s1, entry, spec_exit, first);
