@@ -171,7 +171,12 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
         if (active) {
             const int q = p - d;
             const int off = qr ? bestL - 7 : k;
-            const int lq = link[sk(q)];  // next chain member, loaded with the compare words
+            // next chain member, loaded with the compare words every iteration
+            // (volatile: kept off the candidate-change path's latency)
+            int lq;
+            asm volatile("ld.volatile.shared.u8 %0, [%1];"
+                         : "=r"(lq)
+                         : "r"((uint32_t)__cvta_generic_to_shared(link + sk(q))));
             const Be8 vq = load8(u, q + off), vp = load8(u, p + off);
             const uint32_t xh = vq.hi ^ vp.hi, xl = vq.lo ^ vp.lo;
             const int fb = __clzll(((uint64_t)xh << 32) | xl) >> 3;  // equal leading bytes (<= 8), branch-free
