@@ -12,18 +12,21 @@ BENCH_DIST_BACKEND=gloo timeout 600 python -m torch.distributed.run --nnodes=1 -
    > gpurun_out/bench_n2gloo_$TAG.json 2> gpurun_out/bench_n2gloo_$TAG.err
 ncu --metrics gpu__time_duration.sum --clock-control none -c 200 --csv \
     --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e \
-    --no-decompress > /dev/null 2>&1
+    --no-decompress --no-versions > /dev/null 2>&1
 ncu --metrics gpu__time_duration.sum --clock-control none -c 200 --csv \
     --log-file gpurun_out/launches_dec_$TAG.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-e2e \
-    > /dev/null 2>&1
+    --no-versions > /dev/null 2>&1
 for cfg in c2_csource_128m c4_random_1g c3_runs20_1g; do
   ncu --set full --clock-control none --import-source on -k regex:chunk_kernel -s 1 -c 1 \
       -o gpurun_out/full_${cfg}_$TAG python bench.py --config $cfg --steps 1 --warmup 1 --no-cpu-baseline --no-e2e \
-      > /dev/null 2>&1
+      --no-versions > /dev/null 2>&1
 done
 for k in walk_kernel decode_kernel; do
   ncu --set full --clock-control none --import-source on -k regex:$k -s 1 -c 1 \
       -o gpurun_out/full_${k}_c2_$TAG python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-e2e \
-      > /dev/null 2>&1
+      --no-versions > /dev/null 2>&1
 done
+python bench.py --config c5_tarmix_64g --steps 3 --warmup 3 --no-cpu-baseline > gpurun_out/bench_c5_$TAG.json 2>&1
+python bench.py --config c3_runs20_1g --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/bench_c3_$TAG.json 2>&1
+python bench.py --config c4_random_1g --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/bench_c4_$TAG.json 2>&1
 tail -c 3000 gpurun_out/bench_full_$TAG.json; echo; tail -3 gpurun_out/bench_n2gloo_$TAG.json; tail -c 600 gpurun_out/bench_ref_$TAG.json
