@@ -84,6 +84,7 @@ culzss_status check_params(const culzss_params *p, Geometry *g) {
     g->S = p->chunk_size;
     g->W = p->window;
     g->F = p->max_match;
+    set_packing(g);
     return CULZSS_OK;
 }
 

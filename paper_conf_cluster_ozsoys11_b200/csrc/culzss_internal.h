@@ -23,7 +23,19 @@ struct Geometry {
     uint32_t S, W, F;               // chunk, window, max match (MIN is 3)
     uint32_t V = 0;                 // kernel version: 0 = lazy hash-chain search,
                                     // 2 = the paper's V2 all-position search
+    uint32_t K = 1;                 // chunks per warp pair: 4096 / S for S in {64, 128, ..., 2048},
+                                    // else 1 (small chunks packed into one 4096-position buffer)
+    uint32_t smask = 4095;          // S - 1 when K > 1: position p's chunk is [p & ~smask, +S)
 };
+// Chunk packing for the fused kernel: chunks of S = 64 .. 2048
+// (powers of two) share one warp pair, K = 4096 / S of them, so every 64-position
+// walk segment lies inside one chunk.
+inline void set_packing(Geometry *g) {
+    const uint32_t S = g->S;
+    const bool pack = S >= 64 && S <= 2048 && (S & (S - 1)) == 0;
+    g->K = pack ? 4096 / S : 1;
+    g->smask = pack ? S - 1 : 4095;
+}
 
 // Per-warp shared memory.  Per-position arrays use a SKEWED layout: 4 pad
 // bytes after every 128-position segment, so that the 32 lanes (one segment
@@ -84,4 +96,10 @@ uint64_t decode_scratch_bytes(uint64_t C);
 
 void count_launch(int k = 1);
 
+}  // namespace culzss
+
+namespace culzss {
+// packed small chunks: K buckets of bucket_stride(S) bytes must fit in the ld area (S = 64 is the largest)
+static_assert((kChunkMax / 64) * (((64 * 9 + 7) / 8 + 15) / 16 * 16) <= sizeof(WarpSmem::a.u.w.ld), "packed buckets fit in ld");
+static_assert((kChunkMax / 128) * (((128 * 9 + 7) / 8 + 15) / 16 * 16) <= sizeof(WarpSmem::a.u.w.ld), "packed buckets fit in ld");
 }  // namespace culzss

@@ -267,11 +267,13 @@ __device__ __forceinline__ uint32_t v2_run(const uint32_t *cw, int p, int d, uin
     return (uint32_t)min(L, cap);
 }
 
-__device__ void v2_search_all(const uint32_t *cw, uint16_t *ld, int m, int W, int F, int half, int lane) {
+__device__ void v2_search_all(const uint32_t *cw, uint16_t *ld, int m, int W, int F, int half, int lane,
+                              int smask) {
 #pragma unroll 1
     for (int p = half; p < m; p += kWarpsPerChunk) {
-        const int cap = min(F, m - p);
-        const int dmax = min(W, p);
+        // window and lookahead stay inside p's chunk [p & ~smask, +S)
+        const int cap = min(F, min((p | smask) + 1, m) - p);
+        const int dmax = min(W, p & smask);
         uint32_t best = 0;
         if (cap >= 3) {
             const uint32_t p0 = load4(cw, p);  // same word for every lane (broadcast)
@@ -299,7 +301,7 @@ __device__ __forceinline__ void pair_sync(int id) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(kWalkLanes) : "memory");
 }
 
-template <int MODE, bool SMALLW, bool V2>
+template <int MODE, bool SMALLW, bool V2, bool PACK>
 __global__ void __launch_bounds__(kChunksPerCta * kWalkLanes, kCtasPerSm)
 chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__restrict__ bucket,
              uint32_t *__restrict__ sizes, void *__restrict__ dbg) {
@@ -311,10 +313,13 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     const int bar = 1 + pair;                      // named barrier of the warp pair
     WarpSmem &sm = reinterpret_cast<WarpSmem *>(smem_raw)[pair];
     const uint64_t C = (n + g.S - 1) / g.S;
-    const uint64_t c = (uint64_t)blockIdx.x * kChunksPerCta + pair;
+    // the pair's chunks [c, c + K): K = 1 (S > 2048 or not a power of two) or
+    // 4096 / S small chunks packed back to back into one 4096-position buffer
+    const uint64_t c = ((uint64_t)blockIdx.x * kChunksPerCta + pair) * g.K;
     if (c >= C) return;  // both warps of the pair leave together
     const uint64_t start = c * g.S;
-    const int m = (int)min((uint64_t)g.S, n - start);
+    const int m = (int)min((uint64_t)g.K * g.S, n - start);
+    const int smask = PACK ? (int)g.smask : 4095;  // !PACK: one chunk, no inner bounds
     const int W = g.W, F = g.F;
     const uint8_t *src = in + start;
     uint8_t *cb = reinterpret_cast<uint8_t *>(sm.cw);
@@ -403,7 +408,14 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                                 *e = (uint8_t)(p + j);
                             }
                             const uint32_t D = __vsub4(__vadd4(((uint32_t)p & 0xFFu) * 0x01010101u, 0x03020100u), E);
-                            lw = D & __vcmpleu4(D, w4);  // distance, or 0 past the window
+                            // at most W, and never before the chunk start (packed
+                            // small chunks; a 4-group lies in one chunk)
+                            uint32_t lim = w4;
+                            if (PACK) {
+                                const uint32_t rel = (uint32_t)min(p & smask, 252);
+                                lim = __vminu4(w4, __vadd4(rel * 0x01010101u, 0x03020100u));
+                            }
+                            lw = D & __vcmpleu4(D, lim);  // distance, or 0 past the window
                         } else {
 #pragma unroll
                             for (int j = 0; j < 4; j++) {
@@ -411,7 +423,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                                 uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(key));
                                 const uint32_t dist = (uint32_t)(p + j + kTabBias) - *e;
                                 *e = (uint16_t)(p + j + kTabBias);
-                                lw |= (dist <= (uint32_t)W ? dist : 0u) << (8 * j);
+                                const bool ok = dist <= (uint32_t)W && (!PACK || dist <= (uint32_t)((p + j) & smask));
+                                lw |= (ok ? dist : 0u) << (8 * j);
                             }
                         }
                         *reinterpret_cast<uint32_t *>(link + sk(p)) = lw;
@@ -429,7 +442,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     pair_sync(bar);  // tab is dead from here on
     if (V2) {
         // version 2: (L, D) of every position by the warp-cooperative search
-        v2_search_all(sm.cw, sm.a.u.w.ld, m, W, F, half, lane);
+        v2_search_all(sm.cw, sm.a.u.w.ld, m, W, F, half, lane, smask);
         pair_sync(bar);
     }
 
@@ -437,7 +450,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         // every position, for per-position parity (a2)
         uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
         for (int p = t64; p < m; p += kWalkLanes) {
-            const uint32_t t = V2 ? (uint32_t)sm.a.u.w.ld[sk2(p)] : eval_pos(sm.cw, link, p, m, W, F);
+            const uint32_t t = V2 ? (uint32_t)sm.a.u.w.ld[sk2(p)]
+                                  : eval_pos(sm.cw, link, p, min((p | smask) + 1, m), W, F);
             LD[2 * p] = (uint8_t)(t == kLit ? 0 : (t & 0xFF) + 3);
             LD[2 * p + 1] = (uint8_t)(t == kLit ? 0 : t >> 8);
         }
@@ -447,6 +461,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     // ---------------- a3: lazy greedy walk, speculative per 64-segment -----
     const int s0 = t64 * kWSeg;
     const int s1 = min(s0 + kWSeg, m);  // <= s0 for lanes past the chunk end
+    const int ce = PACK ? min((s0 | smask) + 1, m) : m;  // end of the segment's chunk (matches stop there)
     uint16_t *ld = sm.a.u.w.ld;
     uint32_t *ucw = sm.a.u.w.ucw;
     if (!V2) {
@@ -484,7 +499,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     pair_sync(bar);
     bool anym = true;  // the speculative path holds a match (V2: not tracked)
     const uint64_t cm = ((uint64_t)rc0 << 32) | rc1;
-    const int spec_exit = V2 ? v2_jump(ld, s0, s1) : walk_spec(ucw, link, cm, ld, m, W, F, s0, s1, anym);
+    const int spec_exit = V2 ? v2_jump(ld, s0, s1) : walk_spec(ucw, link, cm, ld, ce, W, F, s0, s1, anym);
     int exitp = spec_exit;
     int cur = s0;
     bool first = true;
@@ -512,7 +527,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         par ^= 1;
         if (chg) {
             exitp = V2 ? v2_jump(ld, entry, s1)
-                       : walk_fix(sm.cw, link, cm, ld, m, W, F, s0, s1, entry, spec_exit, first);
+                       : walk_fix(sm.cw, link, cm, ld, ce, W, F, s0, s1, entry, spec_exit, first);
             first = false;
             cur = entry;
         }
@@ -625,16 +640,30 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         total += v;
     }
     incl += before;
-    const int excl = incl - nbits;
-    const int nwords = (total + 31) >> 5;
+    int excl = incl - nbits;
+    const uint64_t stride = bucket_stride(g.S);
+    const int kk = (m + (int)g.S - 1) / (int)g.S;  // chunks in this pair
+    int cbits = total, cword = 0;                  // this lane's chunk: total bits, first payload word
+    if (PACK) {
+        // packed chunks: a chunk's lanes are lpc consecutive lanes of one warp;
+        // bit offsets restart at each chunk, whose payload words start at its
+        // bucket offset in ow (the same layout as the buckets in HBM)
+        const int lpc = (int)g.S / kWSeg;
+        const int first = lane & ~(lpc - 1);
+        const int cbase = __shfl_sync(kFull, excl, first);
+        cbits = __shfl_sync(kFull, excl + nbits, first + lpc - 1) - cbase;
+        excl -= cbase;
+        cword = (t64 / lpc) * (int)(stride / 4);
+    }
+    const int nwords = PACK ? kk * (int)(stride / 4) : ((total + 31) >> 5) + 1;
     uint32_t *ow = reinterpret_cast<uint32_t *>(ld);  // ld is dead: payload words
-    for (int i = t64; i < nwords + 1; i += kWalkLanes) ow[i] = 0;
+    for (int i = t64; i < nwords; i += kWalkLanes) ow[i] = 0;
     pair_sync(bar);
     {
         // shift the lane's staged words to bit offset excl; output words shared
         // with the neighbouring lanes (first, last, spill) are OR-ed atomically
         const int sh = excl & 31;
-        const int base = excl >> 5;
+        const int base = cword + (excl >> 5);
         const int nsw = (nbits + 31) >> 5;
         uint32_t prev = 0;
 #pragma unroll 1
@@ -651,12 +680,13 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     }
     pair_sync(bar);
 
-    // payload -> bucket c (bytes in stream order: big-endian words)
-    const int nbytes = (total + 7) >> 3;
-    const uint64_t stride = bucket_stride(g.S);
+    // payload(s) -> bucket c.. (bytes in stream order: big-endian words); with
+    // packed chunks the kk buckets are contiguous in HBM as in ow
+    const int nbytes = (cbits + 7) >> 3;
     uint4 *dst = reinterpret_cast<uint4 *>(bucket + c * stride);
     const uint4 *o4 = reinterpret_cast<const uint4 *>(ow);
-    for (int i = t64; i < (nbytes + 15) >> 4; i += kWalkLanes) {
+    const int n16 = PACK ? kk * (int)(stride / 16) : (nbytes + 15) >> 4;
+    for (int i = t64; i < n16; i += kWalkLanes) {
         uint4 v = o4[i];
         v.x = __byte_perm(v.x, 0, 0x0123);
         v.y = __byte_perm(v.y, 0, 0x0123);
@@ -664,10 +694,15 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         v.w = __byte_perm(v.w, 0, 0x0123);
         dst[i] = v;
     }
-    if (t64 == 0) sizes[c] = (uint32_t)nbytes;
+    if (PACK) {
+        const int lpc = (int)g.S / kWSeg;
+        if ((t64 & (lpc - 1)) == 0 && t64 / lpc < kk) sizes[c + t64 / lpc] = (uint32_t)nbytes;
+    } else if (t64 == 0) {
+        sizes[c] = (uint32_t)nbytes;
+    }
 }
 
-template <int MODE, bool SMALLW, bool V2>
+template <int MODE, bool SMALLW, bool V2, bool PACK>
 cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *bucket,
                         uint32_t *sizes, void *dbg, cudaStream_t st) {
     const uint64_t C = (n + g.S - 1) / g.S;
@@ -675,13 +710,14 @@ cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *buck
     const size_t smem = sizeof(WarpSmem) * kChunksPerCta;
     static bool attr_set = false;  // benign race: idempotent
     if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(chunk_kernel<MODE, SMALLW, V2>,
+        cudaError_t e = cudaFuncSetAttribute(chunk_kernel<MODE, SMALLW, V2, PACK>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         attr_set = true;
     }
-    const uint64_t blocks = (C + kChunksPerCta - 1) / kChunksPerCta;
-    chunk_kernel<MODE, SMALLW, V2><<<(unsigned)blocks, kChunksPerCta * kWalkLanes, smem, st>>>(in, n, g, bucket,
+    const uint64_t pairs = (C + g.K - 1) / g.K;
+    const uint64_t blocks = (pairs + kChunksPerCta - 1) / kChunksPerCta;
+    chunk_kernel<MODE, SMALLW, V2, PACK><<<(unsigned)blocks, kChunksPerCta * kWalkLanes, smem, st>>>(in, n, g, bucket,
                                                                                             sizes, dbg);
     count_launch();
     return cudaGetLastError();
@@ -690,9 +726,15 @@ cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *buck
 template <int MODE>
 cudaError_t launch_w(const uint8_t *in, uint64_t n, Geometry g, uint8_t *bucket, uint32_t *sizes,
                      void *dbg, cudaStream_t st) {
-    if (g.V == 2) return launch_mode<MODE, false, true>(in, n, g, bucket, sizes, dbg, st);
-    return g.W <= 128 ? launch_mode<MODE, true, false>(in, n, g, bucket, sizes, dbg, st)
-                      : launch_mode<MODE, false, false>(in, n, g, bucket, sizes, dbg, st);
+    const bool pack = g.K > 1;
+    if (g.V == 2)
+        return pack ? launch_mode<MODE, false, true, true>(in, n, g, bucket, sizes, dbg, st)
+                    : launch_mode<MODE, false, true, false>(in, n, g, bucket, sizes, dbg, st);
+    if (g.W <= 128)
+        return pack ? launch_mode<MODE, true, false, true>(in, n, g, bucket, sizes, dbg, st)
+                    : launch_mode<MODE, true, false, false>(in, n, g, bucket, sizes, dbg, st);
+    return pack ? launch_mode<MODE, false, false, true>(in, n, g, bucket, sizes, dbg, st)
+                : launch_mode<MODE, false, false, false>(in, n, g, bucket, sizes, dbg, st);
 }
 
 }  // namespace

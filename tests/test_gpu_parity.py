@@ -349,3 +349,36 @@ def test_full_size_configs(env, cfg):
     assert torch.equal(x, y)
     del y, s, x
     torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("S", [64, 128, 256, 512, 1024, 2048])
+@pytest.mark.parametrize("W,F", [(128, 128), (32, 258), (255, 200), (1, 3)])
+def test_packed_small_chunks(env, S, W, F):
+    """Chunks of S = 64..2048 are packed 4096 / S to a warp pair: every
+    window, lookahead and bit stream must still stop at its own chunk's
+    bounds.  Ragged totals leave a partial last pair and a partial last chunk."""
+    torch, culzss = env
+    for kind in ("english", "runs20", "period20", "tarmix"):
+        n = 3 * 4096 + 5 * S + S // 3 + 1
+        x = datagen.generate(kind, n, seed=S + W)
+        assert gpu_stream(env, x, S=S, W=W, F=F) == O.compress(x, S=S, W=W, F=F), kind
+
+
+@pytest.mark.parametrize("S", [64, 256, 2048])
+def test_packed_small_chunks_match_and_tokens(env, S):
+    """Rows a2/a3 with packed chunks: per-position (L, D) and parse tokens
+    per chunk, versions 0 and 2."""
+    torch, culzss = env
+    x = datagen.generate("csource", 2 * 4096 + 3 * S + 7, seed=S)
+    for version in (0, 2):
+        p = culzss.Params.make(S=S, version=version)
+        L, D = culzss.match_search(dev(torch, x), p)
+        L, D = L.cpu().numpy(), D.cpu().numpy()
+        tok = culzss.parse_tokens(dev(torch, x), p).cpu().numpy().astype(np.int64) & 0xFFFFFFFF
+        for c in range((x.size + S - 1) // S):
+            chunk = x[c * S:(c + 1) * S]
+            eL, eD = O.match_all(chunk)
+            np.testing.assert_array_equal(L[c * S:c * S + chunk.size], eL, err_msg=f"v{version} c{c}")
+            np.testing.assert_array_equal(D[c * S:c * S + chunk.size], eD, err_msg=f"v{version} c{c}")
+            np.testing.assert_array_equal(tok[c * S:c * S + chunk.size],
+                                          expand_tokens(O.tokens_chunk(chunk), chunk.size))
