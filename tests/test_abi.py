@@ -29,7 +29,8 @@ def test_header_declares_expected_entry_points():
     syms = header_symbols()
     for s in ("culzss_compress", "culzss_decompress", "culzss_compress_chunks", "culzss_write_header",
               "culzss_max_compressed_size", "culzss_default_params", "culzss_status_string",
-              "culzss_match_search", "culzss_parse_tokens", "culzss_compress_host"):
+              "culzss_match_search", "culzss_parse_tokens", "culzss_compress_host",
+              "culzss_decompress_chunks"):
         assert s in syms
 
 
@@ -71,6 +72,10 @@ def test_no_cpu_fallback_without_device(culzss):
     buf = (ctypes.c_uint8 * 64)()
     st = culzss.lib().culzss_compress(ctypes.cast(buf, ctypes.c_void_p), 64, ctypes.cast(buf, ctypes.c_void_p),
                                       ctypes.byref(on), None, None)
+    assert st == culzss.ERR_NO_DEVICE
+    sizes = (ctypes.c_uint32 * 1)()
+    st = culzss.lib().culzss_decompress_chunks(ctypes.cast(buf, ctypes.c_void_p), 8, ctypes.cast(sizes, ctypes.c_void_p),
+                                               64, ctypes.cast(buf, ctypes.c_void_p), None, None)
     assert st == culzss.ERR_NO_DEVICE
 
 
