@@ -143,3 +143,15 @@ def test_mutated_streams_never_crash(raw, seed, nmut):
     assert st_ in (O.OK, O.ERR_CORRUPT)
     if st_ == O.OK:
         assert len(out) == struct.unpack("<Q", bytes(s[16:24]))[0]
+
+
+@pytest.mark.parametrize("S,W,F,k", [(64, 128, 128, 3), (64, 255, 258, 2), (128, 128, 20, 4), (512, 64, 128, 3)])
+def test_small_chunks_window_beyond_chunk(S, W, F, k):
+    """Chunks smaller than the window (the packed GPU geometry's case): the
+    window never reaches before the chunk start (R5) and the lookahead stops
+    at its end, against the independent definition."""
+    rng = np.random.default_rng(S + W + F + k)
+    for _ in range(3):
+        n = int(rng.integers(3 * S, 3 * S + 200))
+        s = bytes(rng.integers(0, k, size=n, dtype=np.uint8).tolist())
+        assert O.compress(s, S=S, W=W, F=F) == ref_stream(s, S, W, F)
