@@ -165,7 +165,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
         cap = min(F, m - p);
     }
     int k = 0, bestL = 2, bestD = 0;
-    bool qr = false;
+    int qr = 0;  // reject-test mode (int: no byte-register repacking)
 #pragma unroll 1
     while (__any_sync(kFull, active)) {
         if (active) {
@@ -186,7 +186,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
             bestL = upd ? L : bestL;
             bestD = upd ? d : bestD;
             k = qr ? 0 : k + 8;
-            qr = qr && fb < 8;
+            qr = qr && fb < 8 ? 1 : 0;
             bool tok_done = false;
             if (cand_done) {
                 const int l2 = bestL == cap ? 0 : lq;
@@ -194,7 +194,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
                 tok_done = l2 == 0 || nd > W;
                 d = nd;
                 k = 0;
-                qr = bestL >= 8;
+                qr = bestL >= 8 ? 1 : 0;
             }
             if (tok_done) {
                 lds[p] = (uint16_t)(bestD ? (bestD << 8) | (bestL - 3) : kLit);
@@ -208,7 +208,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
                 bestL = 2;
                 bestD = 0;
                 k = 0;
-                qr = false;
+                qr = 0;
             }
         }
     }
