@@ -85,8 +85,9 @@ __device__ __forceinline__ Be8 load8(const uint32_t *__restrict__ u, int x) {
 // p >= s1 already).  cm: candidate bits of positions s0..s0+63, position
 // s0+i at bit 63-i (reversed: next = count of leading zeros)
 __device__ __forceinline__ int next_cand(uint64_t cm, int p, int s0, int s1) {
-    if (p >= s1) return p;
-    return min(p + __clzll(cm << (p - s0)), s1);  // clz(0) = 64: past the segment
+    // branch-free: for p >= s1 the min gives s1 and the max restores p
+    const int nc = min(p + __clzll(cm << min(p - s0, 63)), s1);  // clz(0) = 64: past the segment
+    return max(nc, p);
 }
 
 __device__ __forceinline__ bool is_cand(uint64_t cm, int o) { return (cm << o) >> 63; }
