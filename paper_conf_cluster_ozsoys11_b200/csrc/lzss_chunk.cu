@@ -592,33 +592,40 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                 put(((bytes & 0xFFu) << 9) | ((bytes >> 8) & 0xFFu), 18);
                 put((((bytes >> 16) & 0xFFu) << 9) | (bytes >> 24), 18);
             }
-        } else
-#pragma unroll 1
-        for (int i = max(0, (cov - s0) >> 2); i < ng; i = max(i + 1, (cov - s0) >> 2)) {
+        } else {
             // groups wholly inside a match are skipped.  Positions are
             // combined in pairs in 32 bits first: a pair is at most a literal
             // and a match (26 bits), since a match covers the next position.
-            const uint32_t bytes = cbw[i];
-            const uint32_t t01 = ldw[2 * i], t23 = ldw[2 * i + 1];
-            uint32_t pv = 0;
-            int pn = 0;
+            // Only a chunk's last lane can have a partial last group: full
+            // groups skip the segment-end test.
+            auto group = [&](int i, bool chk) {
+                const uint32_t bytes = cbw[i];
+                const uint32_t t01 = ldw[2 * i], t23 = ldw[2 * i + 1];
+                uint32_t pv = 0;
+                int pn = 0;
 #pragma unroll
-            for (int j = 0; j < 4; j++) {
-                const int p = s0 + 4 * i + j;
-                const uint32_t t = (j < 2 ? t01 : t23) >> (16 * (j & 1)) & 0xFFFFu;
-                const bool on = p >= cov && p < s1;
-                const bool mt = on && t >= 0x100;
-                const int nb = mt ? 17 : (on ? 9 : 0);
-                const uint32_t val = mt ? t + (0x10000u - 0x100u) : (on ? (bytes >> (8 * j)) & 0xFFu : 0u);  // 1|D-1|L-3
-                cov = mt ? p + (int)(t & 0xFF) + 3 : cov;
-                pv = (pv << nb) | val;
-                pn += nb;
-                if (j & 1) {
-                    put(pv, pn);
-                    pv = 0;
-                    pn = 0;
+                for (int j = 0; j < 4; j++) {
+                    const int p = s0 + 4 * i + j;
+                    const uint32_t t = (j < 2 ? t01 : t23) >> (16 * (j & 1)) & 0xFFFFu;
+                    const bool on = p >= cov && (!chk || p < s1);
+                    const bool mt = on && t >= 0x100;
+                    const int nb = mt ? 17 : (on ? 9 : 0);
+                    const uint32_t val = mt ? t + (0x10000u - 0x100u) : (on ? (bytes >> (8 * j)) & 0xFFu : 0u);  // 1|D-1|L-3
+                    cov = mt ? p + (int)(t & 0xFF) + 3 : cov;
+                    pv = (pv << nb) | val;
+                    pn += nb;
+                    if (j & 1) {
+                        put(pv, pn);
+                        pv = 0;
+                        pn = 0;
+                    }
                 }
-            }
+            };
+            const int ngf = (s1 - s0) >> 2;  // full groups
+            int i = max(0, (cov - s0) >> 2);
+#pragma unroll 1
+            for (; i < ngf; i = max(i + 1, (cov - s0) >> 2)) group(i, false);
+            if (i == ngf && ngf < ng) group(i, true);
         }
         const int nw = (int)(sp - stage);
         nbits = 32 * nw + nacc;
