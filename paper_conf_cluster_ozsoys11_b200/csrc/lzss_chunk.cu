@@ -673,16 +673,24 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         const int sh = excl & 31;
         const int base = cword + (excl >> 5);
         const int nsw = (nbits + 31) >> 5;
-        uint32_t prev = 0;
+        if (nsw) {
+            // word i of the output = bits of staged words i-1, i shifted by sh
+            // (funnel shift: sh = 0 gives the word itself); the first and last
+            // (and the spill word) are shared with neighbours
+            uint32_t prev = stage[0];
+            atomicOr(&ow[base], prev >> sh);
 #pragma unroll 1
-        for (int i = 0; i < nsw; i++) {
-            const uint32_t v = stage[i];
-            const uint32_t o = sh ? (prev << (32 - sh)) | (v >> sh) : v;
-            if (i == 0 || i == nsw - 1) atomicOr(&ow[base + i], o); else ow[base + i] = o;
-            prev = v;
-        }
-        if (sh && nsw) {
-            const uint32_t o = prev << (32 - sh);
+            for (int i = 1; i < nsw - 1; i++) {
+                const uint32_t v = stage[i];
+                ow[base + i] = __funnelshift_r(v, prev, sh);
+                prev = v;
+            }
+            if (nsw > 1) {
+                const uint32_t v = stage[nsw - 1];
+                atomicOr(&ow[base + nsw - 1], __funnelshift_r(v, prev, sh));
+                prev = v;
+            }
+            const uint32_t o = sh ? prev << (32 - sh) : 0u;
             if (o) atomicOr(&ow[base + nsw], o);
         }
     }
