@@ -26,7 +26,7 @@ for k in walk_kernel decode_kernel; do
       -o gpurun_out/full_${k}_c2_$TAG python bench.py --steps 1 --warmup 1 --no-cpu-baseline --no-e2e \
       --no-versions > /dev/null 2>&1
 done
-python bench.py --config c5_tarmix_64g --steps 3 --warmup 3 --no-cpu-baseline > gpurun_out/bench_c5_$TAG.json 2>&1
-python bench.py --config c3_runs20_1g --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/bench_c3_$TAG.json 2>&1
-python bench.py --config c4_random_1g --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/bench_c4_$TAG.json 2>&1
+python bench.py --config c5_tarmix_64g --steps 3 --warmup 3 > gpurun_out/bench_c5_$TAG.json 2>&1
+python bench.py --config c3_runs20_1g --steps 5 --warmup 3 > gpurun_out/bench_c3_$TAG.json 2>&1
+python bench.py --config c4_random_1g --steps 5 --warmup 3 > gpurun_out/bench_c4_$TAG.json 2>&1
 tail -c 3000 gpurun_out/bench_full_$TAG.json; echo; tail -3 gpurun_out/bench_n2gloo_$TAG.json; tail -c 600 gpurun_out/bench_ref_$TAG.json
