@@ -10,12 +10,14 @@ echo "Captured with \`tools/profile_round.sh $TAG\` (ncu --set full --clock-cont
 echo
 echo "Bench lines of the same build (no profiler, same box, \`gpurun_out/bench_*_$TAG.json\`):"
 echo
-echo "| config | compress GB/s | ratio | chunk_kernel ms | roofline frac (alu) | decompress GB/s | e2e GB/s | version 2 GB/s | SM MHz / throttle |"
-echo "|---|---|---|---|---|---|---|---|---|"
+echo "| config | compress GB/s | ratio | chunk_kernel ms | roofline frac (alu) | decompress GB/s | e2e GB/s | version 2 GB/s | CPU oracle GB/s (threads) | SM MHz / throttle |"
+echo "|---|---|---|---|---|---|---|---|---|---|"
 for f in bench_full_$TAG bench_c3_$TAG bench_c4_$TAG bench_c5_$TAG; do python -c "
 import json; d=json.loads(open('gpurun_out/$f.json').read().strip().splitlines()[-1])
 v=d.get('versions',{}).get('2',{}).get('value')
-print('| %s | %.1f | %.4f | %.3f | %.3f | %.1f | %.1f | %s | %s %s |' % (d['config']['workload'].split(':')[0], d['value'], d['ratio'], d['kernels_ms']['chunk'], d['roofline']['frac'], d['decompress']['value'], d['e2e']['value'], '%.2f'%v if v else '-', d['clocks']['sm_mhz'], d['clocks']['reasons'] or 'none'))"; done
+c=d.get('cpu_baseline')
+cs='%.3f (%d)' % (c['value'], c['cores']) if c else '-'
+print('| %s | %.1f | %.4f | %.3f | %.3f | %.1f | %.1f | %s | %s | %s %s |' % (d['config']['workload'].split(':')[0], d['value'], d['ratio'], d['kernels_ms']['chunk'], d['roofline']['frac'], d['decompress']['value'], d['e2e']['value'], '%.2f'%v if v else '-', cs, d['clocks']['sm_mhz'], d['clocks']['reasons'] or 'none'))"; done
 python -c "
 import json; d=json.loads(open('gpurun_out/bench_full_$TAG.json').read().strip().splitlines()[-1]); c=d['cpu_baseline']
 print(); print('CPU oracle beside it (c2, same run): %.3f GB/s on %d threads (%s).' % (c['value'], c['cores'], c['sample']))
