@@ -372,7 +372,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + (SMALLW ? 512 * lane : 2 * lane);
         if (b0 < m) {
             // the W positions before the segment (pre-insert, no links)
-#pragma unroll 1
+#pragma unroll 4
             for (int q = max(0, b0 - W) & ~3; q < b0; q += 4) {
                 const uint32_t w0 = sm.cw[sk(q) >> 2], w1 = sm.cw[(sk(q) >> 2) + 1];
 #pragma unroll
