@@ -470,7 +470,9 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         // unskew the chunk for the walks' compares
         uint4 *l4 = reinterpret_cast<uint4 *>(ld);
         const uint4 z = make_uint4(0, 0, 0, 0);
+#pragma unroll 4
         for (int i = t64; i < (int)(sizeof(sm.a.u.w.ld) / 16); i += kWalkLanes) l4[i] = z;
+#pragma unroll 4
         for (int j = t64; j < kUcwWords; j += kWalkLanes) ucw[j] = __byte_perm(sm.cw[j + (j >> 5)], 0, 0x0123);
     }
     // candidate mask: bit i = position s0 + i (< s1) has a chain link
@@ -665,6 +667,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     }
     const int nwords = PACK ? kk * (int)(stride / 4) : ((total + 31) >> 5) + 1;
     uint32_t *ow = reinterpret_cast<uint32_t *>(ld);  // ld is dead: payload words
+#pragma unroll 4
     for (int i = t64; i < nwords; i += kWalkLanes) ow[i] = 0;
     pair_sync(bar);
     {
