@@ -327,10 +327,18 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     uint8_t *link = sm.a.link;
 
     // ---------------- a1: stage the chunk (16-byte coalesced loads) --------
+    // a full chunk overwrites every data byte: only the zero tail (read by
+    // the 8-byte compares past the end) needs clearing, and no barrier has to
+    // order the clearing before the data stores
+    const bool full = m == kChunkMax;
     {
         uint4 *z4 = reinterpret_cast<uint4 *>(sm.cw);
         const uint4 z = make_uint4(0, 0, 0, 0);
-        for (int i = t64; i < (int)(sizeof(sm.cw) / 16); i += kWalkLanes) z4[i] = z;
+        if (!full) {
+            for (int i = t64; i < (int)(sizeof(sm.cw) / 16); i += kWalkLanes) z4[i] = z;
+        } else if (t64 == 0) {
+            z4[sizeof(sm.cw) / 16 - 1] = z;
+        }
         uint4 *t4 = reinterpret_cast<uint4 *>(sm.a.u.tab);
         // u8 tables: empty = (s0 - 129) mod 256 = 0x7F (even lanes) / 0xFF (odd)
 #pragma unroll 4
@@ -340,11 +348,12 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
             t4[i] = make_uint4(e, e, e, e);
         }
     }
-    pair_sync(bar);
+    if (!full) pair_sync(bar);  // (uniform per pair)
     if ((reinterpret_cast<uintptr_t>(src) & 15) == 0) {
         // a 16-byte group never straddles a 128-position segment
         const int nvec = m >> 4;
         const uint4 *s4 = reinterpret_cast<const uint4 *>(src);
+#pragma unroll 4
         for (int i = t64; i < nvec; i += kWalkLanes) {
             const uint4 v = __ldcs(s4 + i);
             uint32_t *d = sm.cw + (sk(i << 4) >> 2);
