@@ -338,7 +338,9 @@ def main():
         pass
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "warmup": args.warmup, "ms_per_step": ms_per_step,
+        "ms_step_median": statistics.median(step_ms), "ms_step_min": min(step_ms),  # this rank's
+        "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": f"{args.config}: {CONFIG_TEXT[args.config]}", "bytes_per_rank": n,
                    "chunk": 4096, "window": 128, "max_match": 128, "min_match": 3,
