@@ -194,7 +194,7 @@ struct CoreLayout {
 // `wsp`: a CoreLayout-sized device workspace, or null to allocate one on st.
 culzss_status compress_core(const uint8_t *in, uint64_t n, const Geometry &g, uint8_t *pay,
                             uint32_t *table, uint32_t *sizes_out, uint64_t *dev_total,
-                            cudaStream_t st, void *wsp = nullptr) {
+                            cudaStream_t st, void *wsp = nullptr, bool prof = true) {
     const uint64_t C = n_chunks(n, g.S);
     const uint64_t stride = bucket_stride(g.S);
     const CoreLayout lay(C, g.S);
@@ -210,13 +210,13 @@ culzss_status compress_core(const uint8_t *in, uint64_t n, const Geometry &g, ui
     uint64_t *offsets = reinterpret_cast<uint64_t *>(base + offs_off);
     uint64_t *scanws = reinterpret_cast<uint64_t *>(base + ws_off);
 
-    t_prof.rec(1, st);
+    if (prof) t_prof.rec(1, st);
     CK(launch_chunk_kernel(kModeCompress, in, n, g, bucket, sizes, nullptr, st));
-    t_prof.rec(2, st);
+    if (prof) t_prof.rec(2, st);
     CK(launch_scan(sizes, C, offsets, dev_total, scanws, st));
-    t_prof.rec(3, st);
+    if (prof) t_prof.rec(3, st);
     CK(launch_compact(bucket, stride, sizes, offsets, C, pay, table, st));
-    t_prof.rec(4, st);
+    if (prof) t_prof.rec(4, st);
     return CULZSS_OK;
 }
 
@@ -522,7 +522,7 @@ culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host
         CK(cudaMemcpyAsync(din + b0, hin + b0, nb, cudaMemcpyHostToDevice, cs));
         s = compress_core(din + b0, nb, g, dstg + payload_bound(b0, g.S),
                           reinterpret_cast<uint32_t *>(dht + 32) + c0, nullptr, hp.dtot + k, cs,
-                          dcore + (k % kPipeStreams) * core_bytes);
+                          dcore + (k % kPipeStreams) * core_bytes, false);  // no per-group profiling events in the issue loop
         if (s != CULZSS_OK) return s;
         CK(cudaMemcpyAsync(hout + 32 + 4 * c0, dht + 32 + 4 * c0, 4 * (c1 - c0), cudaMemcpyDeviceToHost,
                            cs));
