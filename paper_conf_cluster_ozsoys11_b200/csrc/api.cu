@@ -314,33 +314,33 @@ culzss_status culzss_compress(const void *in, size_t n, void *out, size_t *out_n
     uint8_t *o = static_cast<uint8_t *>(out);
     uint64_t *hw = host_word();
     if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
-    t_prof.reset();
-    t_prof.rec(0, st);
-    {
-        cudaError_t e = launch_header(o, n, g, st);
-        if (e != cudaSuccess) return cuda_fail(e);
-    }
     if (n == 0) {
+        t_prof.reset();
+        CK(launch_header(o, n, g, st));
         CK(cudaStreamSynchronize(st));
         *out_n = 32;
         return CULZSS_OK;
     }
-    uint64_t *dev_total = nullptr;
-    CK(cudaMallocAsync(&dev_total, 8, st));
+    // workspace (core layout + the device total) is taken from the stream-
+    // ordered pool before the call's first event: the device-timed region
+    // holds the kernels and the 8-byte read-back, not host-side allocation
+    const CoreLayout lay(C, g.S);
+    const uint64_t tot_off = (lay.total + 255) / 256 * 256;
+    Workspace ws(st);
+    CK(ws.alloc(tot_off + 256));
+    uint64_t *dev_total = reinterpret_cast<uint64_t *>(static_cast<uint8_t *>(ws.p) + tot_off);
+    t_prof.reset();
+    t_prof.rec(0, st);
+    CK(launch_header(o, n, g, st));
     s = compress_core(static_cast<const uint8_t *>(in), n, g, o + 32 + 4 * C,
-                      reinterpret_cast<uint32_t *>(o + 32), nullptr, dev_total, st);
-    if (s == CULZSS_OK) {
-        cudaError_t e = cudaMemcpyAsync(hw, dev_total, 8, cudaMemcpyDeviceToHost, st);
-        t_prof.rec(5, st);
-        if (e == cudaSuccess) e = cudaFreeAsync(dev_total, st);
-        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-        if (e != cudaSuccess) return cuda_fail(e);
-        prof_finish_compress();
-        *out_n = (size_t)(32 + 4 * C + *hw);
-        return CULZSS_OK;
-    }
-    cudaFreeAsync(dev_total, st);
-    return s;
+                      reinterpret_cast<uint32_t *>(o + 32), nullptr, dev_total, st, ws.p);
+    if (s != CULZSS_OK) return s;
+    CK(cudaMemcpyAsync(hw, dev_total, 8, cudaMemcpyDeviceToHost, st));
+    t_prof.rec(5, st);
+    CK(cudaStreamSynchronize(st));
+    prof_finish_compress();
+    *out_n = (size_t)(32 + 4 * C + *hw);
+    return CULZSS_OK;
 }
 
 culzss_status culzss_compress_chunks(const void *in_slice, size_t slice_n, void *payload,
@@ -366,24 +366,23 @@ culzss_status culzss_compress_chunks(const void *in_slice, size_t slice_n, void 
         return CULZSS_ERR_INVALID_ARG;
     uint64_t *hw = host_word();
     if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
-    uint64_t *dev_total = nullptr;
+    // workspace before the first event (see culzss_compress)
+    const CoreLayout lay(n_chunks(slice_n, g.S), g.S);
+    const uint64_t tot_off = (lay.total + 255) / 256 * 256;
+    Workspace ws(st);
+    CK(ws.alloc(tot_off + 256));
+    uint64_t *dev_total = reinterpret_cast<uint64_t *>(static_cast<uint8_t *>(ws.p) + tot_off);
     t_prof.reset();
     t_prof.rec(0, st);
-    CK(cudaMallocAsync(&dev_total, 8, st));
     s = compress_core(static_cast<const uint8_t *>(in_slice), slice_n, g,
-                      static_cast<uint8_t *>(payload), nullptr, chunk_sizes, dev_total, st);
-    if (s == CULZSS_OK) {
-        cudaError_t e = cudaMemcpyAsync(hw, dev_total, 8, cudaMemcpyDeviceToHost, st);
-        t_prof.rec(5, st);
-        if (e == cudaSuccess) e = cudaFreeAsync(dev_total, st);
-        if (e == cudaSuccess) e = cudaStreamSynchronize(st);
-        if (e != cudaSuccess) return cuda_fail(e);
-        prof_finish_compress();
-        *payload_n = (size_t)*hw;
-        return CULZSS_OK;
-    }
-    cudaFreeAsync(dev_total, st);
-    return s;
+                      static_cast<uint8_t *>(payload), nullptr, chunk_sizes, dev_total, st, ws.p);
+    if (s != CULZSS_OK) return s;
+    CK(cudaMemcpyAsync(hw, dev_total, 8, cudaMemcpyDeviceToHost, st));
+    t_prof.rec(5, st);
+    CK(cudaStreamSynchronize(st));
+    prof_finish_compress();
+    *payload_n = (size_t)*hw;
+    return CULZSS_OK;
 }
 
 // Pipelined host-memory compression: the chunks go in groups of ~8 MiB.
