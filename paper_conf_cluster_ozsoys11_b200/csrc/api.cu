@@ -27,7 +27,7 @@ void count_launch(int k) { g_launches.fetch_add((uint64_t)k, std::memory_order_r
 namespace {
 
 thread_local int t_last_cuda_error = 0;
-thread_local bool t_profiling = false;
+thread_local int t_profiling = 0;  // 0 off, 1 call + per-kernel events, 2 call events only
 struct KernelTimes {
     float chunk = -1, scan = -1, compact = -1, decode = -1, call = -1;
 };
@@ -147,6 +147,7 @@ struct Prof {
     bool ready = false;
     void rec(int i, cudaStream_t st) {
         if (!t_profiling) return;
+        if (t_profiling == 2 && i != 0 && i != kN - 1) return;  // nothing between the call's kernels
         if (!ready) {
             for (auto &x : e) cudaEventCreate(&x);
             ready = true;
@@ -210,10 +211,13 @@ culzss_status compress_core(const uint8_t *in, uint64_t n, const Geometry &g, ui
     uint64_t *offsets = reinterpret_cast<uint64_t *>(base + offs_off);
     uint64_t *scanws = reinterpret_cast<uint64_t *>(base + ws_off);
 
+    // the scan's look-back status words are cleared before the chunk kernel,
+    // so nothing but kernels sits between the chunk kernel and the scan
+    CK(cudaMemsetAsync(scanws, 0, scan_workspace_words(C) * sizeof(uint64_t), st));
     if (prof) t_prof.rec(1, st);
     CK(launch_chunk_kernel(kModeCompress, in, n, g, bucket, sizes, nullptr, st));
     if (prof) t_prof.rec(2, st);
-    CK(launch_scan(sizes, C, offsets, dev_total, scanws, st));
+    CK(launch_scan(sizes, C, offsets, dev_total, scanws, st, false));
     if (prof) t_prof.rec(3, st);
     CK(launch_compact(bucket, stride, sizes, offsets, C, pay, table, st));
     if (prof) t_prof.rec(4, st);
@@ -253,7 +257,7 @@ int culzss_device_count(void) {
 
 uint64_t culzss_launch_count(void) { return g_launches.load(); }
 
-void culzss_set_profiling(int enable) { t_profiling = enable != 0; }
+void culzss_set_profiling(int mode) { t_profiling = mode == 1 || mode == 2 ? mode : 0; }
 
 float culzss_last_kernel_ms(const char *name) {
     if (!name) return -1;

@@ -42,6 +42,11 @@ scan_kernel(const uint32_t *__restrict__ sizes, uint64_t C, uint64_t *__restrict
     __shared__ uint64_t warp_sums[kScanThreads / 32];
     __shared__ uint64_t tile_prefix;
     __shared__ uint32_t tile_id;
+    // programmatic dependent launch: the grid may start while its predecessor
+    // (the chunk kernel) drains; wait for its results, and let the compaction
+    // grid get scheduled behind this one
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;");
     if (threadIdx.x == 0) tile_id = (uint32_t)atomicAdd(reinterpret_cast<unsigned long long *>(ws), 1ull);
     __syncthreads();
     const uint64_t tile = tile_id;
@@ -114,6 +119,7 @@ __global__ void __launch_bounds__(256)
 compact_kernel(const uint8_t *__restrict__ bucket, uint64_t stride,
                const uint32_t *__restrict__ sizes, const uint64_t *__restrict__ offsets,
                uint64_t C, uint8_t *__restrict__ out_payload, uint32_t *__restrict__ out_table) {
+    asm volatile("griddepcontrol.wait;" ::: "memory");  // programmatic dependent launch (after the scan)
     const int lane = threadIdx.x & 31;
     const uint64_t c = (uint64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
     if (c >= C) return;
@@ -162,25 +168,45 @@ __global__ void header_kernel(uint8_t *out, uint64_t n, Geometry g) {
 
 uint64_t scan_workspace_words(uint64_t C) { return 1 + (C + kTile - 1) / kTile; }
 
+// Kernel launch with programmatic stream serialization (PDL): the grid may be
+// scheduled before its stream predecessor kernel finishes; the kernel's
+// griddepcontrol.wait orders its reads after that kernel's writes.
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*k)(KArgs...), unsigned grid, unsigned block, cudaStream_t st, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(block);
+    cfg.dynamicSmemBytes = 0;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k, static_cast<KArgs>(args)...);
+}
+
 cudaError_t launch_scan(const uint32_t *sizes, uint64_t C, uint64_t *offsets, uint64_t *total,
-                        uint64_t *ws, cudaStream_t st) {
-    cudaError_t e = cudaMemsetAsync(ws, 0, scan_workspace_words(C) * sizeof(uint64_t), st);
-    if (e != cudaSuccess) return e;
+                        uint64_t *ws, cudaStream_t st, bool zero_ws) {
+    if (zero_ws) {
+        cudaError_t e = cudaMemsetAsync(ws, 0, scan_workspace_words(C) * sizeof(uint64_t), st);
+        if (e != cudaSuccess) return e;
+    }
     if (C == 0) return cudaMemsetAsync(total, 0, sizeof(uint64_t), st);
     const uint64_t ntiles = (C + kTile - 1) / kTile;
-    scan_kernel<<<(unsigned)ntiles, kScanThreads, 0, st>>>(sizes, C, offsets, total, ws);
+    cudaError_t e = launch_pdl(scan_kernel, (unsigned)ntiles, kScanThreads, st, sizes, C, offsets, total, ws);
     count_launch();
-    return cudaGetLastError();
+    return e;
 }
 
 cudaError_t launch_compact(const uint8_t *bucket, uint64_t stride, const uint32_t *sizes,
                            const uint64_t *offsets, uint64_t C, uint8_t *out_payload,
                            uint32_t *out_table, cudaStream_t st) {
     if (C == 0) return cudaSuccess;
-    compact_kernel<<<(unsigned)((C + 7) / 8), 256, 0, st>>>(bucket, stride, sizes, offsets, C,
-                                                            out_payload, out_table);
+    cudaError_t e = launch_pdl(compact_kernel, (unsigned)((C + 7) / 8), 256, st, bucket, stride, sizes, offsets, C,
+                               out_payload, out_table);
     count_launch();
-    return cudaGetLastError();
+    return e;
 }
 
 cudaError_t launch_header(uint8_t *out, uint64_t n, Geometry g, cudaStream_t st) {

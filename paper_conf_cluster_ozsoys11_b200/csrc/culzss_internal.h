@@ -83,7 +83,7 @@ cudaError_t launch_chunk_kernel(int mode, const uint8_t *in, uint64_t n, Geometr
                                 uint8_t *bucket, uint32_t *sizes, void *dbg,
                                 cudaStream_t st);
 cudaError_t launch_scan(const uint32_t *sizes, uint64_t C, uint64_t *offsets,
-                        uint64_t *total, uint64_t *status_ws, cudaStream_t st);
+                        uint64_t *total, uint64_t *status_ws, cudaStream_t st, bool zero_ws = true);
 uint64_t scan_workspace_words(uint64_t C);
 cudaError_t launch_compact(const uint8_t *bucket, uint64_t stride, const uint32_t *sizes,
                            const uint64_t *offsets, uint64_t C, uint8_t *out_payload,

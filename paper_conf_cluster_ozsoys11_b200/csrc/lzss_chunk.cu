@@ -317,6 +317,9 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     // the pair's chunks [c, c + K): K = 1 (S > 2048 or not a power of two) or
     // 4096 / S small chunks packed back to back into one 4096-position buffer
     const uint64_t c = ((uint64_t)blockIdx.x * kChunksPerCta + pair) * g.K;
+    // programmatic dependent launch: the scan grid may be scheduled as soon as
+    // every CTA of this grid has started (it waits for our results itself)
+    asm volatile("griddepcontrol.launch_dependents;");
     if (c >= C) return;  // both warps of the pair leave together
     const uint64_t start = c * g.S;
     const int m = (int)min((uint64_t)g.K * g.S, n - start);

@@ -120,8 +120,10 @@ def launch_count() -> int:
     return int(_lib().culzss_launch_count())
 
 
-def set_profiling(enable: bool) -> None:
-    _lib().culzss_set_profiling(1 if enable else 0)
+def set_profiling(enable, call_only: bool = False) -> None:
+    """enable: per-kernel + call events; call_only: events at the call's start
+    and end only (no event between its kernels)."""
+    _lib().culzss_set_profiling(0 if not enable else (2 if call_only else 1))
 
 
 def last_kernel_ms(name: str) -> float:
