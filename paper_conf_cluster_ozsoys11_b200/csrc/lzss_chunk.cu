@@ -13,32 +13,34 @@
 //   a4  bit-pack  flag 0 + byte | flag 1 + (D-1) + (L-3), MSB first, zero pad
 //                 (PAPER.md:1@4785, @23049-23282; readings R9-R11)
 //
-// B200 design, one warp per chunk, everything in shared memory,
-// lane l owns the 128-position segment [128l, 128l + 128):
-//   * Chain build (a2, part 1).  Each lane inserts the W positions before its
-//     segment and then its own positions, in order, into its own 256-entry
-//     3-gram hash table, recording link[p] = distance to the previous
-//     position with the same hash (0 = none within W).  Every d with
-//     run_d(p) >= 3 shares p's 3-gram, hence its hash, so walking the chain
-//     while the distance stays <= W visits every candidate, nearest first --
-//     the paper's window-offset search without the brute force.  Per-lane
-//     tables make the build a straight-line loop (no intra-warp conflicts).
-//   * Lazy greedy walk (a2 part 2 + a3).  Each lane runs the greedy parse
-//     over its segment from the segment start, evaluating L/D only where the
-//     parse lands -- the V1 "jump over" saving (PAPER.md:1@32329 §V).  The
-//     walk is one flat state machine per lane (each iteration: one candidate
-//     word compare, or the start of a token), so lanes do not serialise on
-//     nested loops; runs of positions with no candidate are emitted as
-//     literals in one step from a 128-bit candidate mask.  Rounds of shuffles
-//     then hand each lane its true entry (the previous lane's exit); a lane
-//     whose entry moved re-walks only until it meets its earlier path, after
-//     which the greedy path is identical.  The result is exactly the serial
-//     greedy parse.
-//   * Bit-pack (a4): per-lane bit counts, warp exclusive scan, each lane ORs
-//     its tokens into the payload words.
-//
-// The match extension compares 4 bytes per step (XOR of two 32-bit words,
-// first differing byte by __ffs): packed byte compares with early out.
+// B200 design: a PAIR of warps per 4 KiB chunk (three pairs per
+// 192-thread CTA, three CTAs per SM), everything in shared memory:
+//   * Chain build (a2, part 1; warp 0).  Lane l owns the 128-position build
+//     segment [128l, 128l + 128) and a private 512-bucket u8 hash table
+//     ([lane][bucket]); it inserts the W positions before its segment, then
+//     its own positions in order, recording link[p] = distance to the previous
+//     position with the same 3-gram hash (0 = none within W; four links per
+//     4-position group formed bytewise with vadd4/vsub4/vcmpleu4).  Every d
+//     with run_d(p) >= 3 shares p's 3-gram, hence its hash, so walking the
+//     chain while the distance stays <= W visits every candidate, nearest
+//     first -- the paper's window-offset search without the brute force.
+//   * Lazy greedy walk (a2 part 2 + a3; both warps).  Walk lane t (0..63) runs
+//     the greedy parse over the 64-position segment [64t, 64t + 64) from its
+//     start, evaluating L/D only where the parse lands -- the V1 "jump over"
+//     saving (PAPER.md:1@32329 §V).  The walk is one flat state machine per
+//     lane: every iteration is one 8-byte compare (big-endian words of an
+//     unskewed chunk copy, equal leading bytes by a 64-bit clz) of one
+//     candidate -- an 8-byte reject test at [bestL-7, bestL] once bestL >= 8,
+//     else an LCP step -- and positions without a candidate are skipped with a
+//     64-bit mask.  Fix-up rounds then hand each lane its true entry (the
+//     previous lane's exit); a lane whose entry moved re-walks only until it
+//     meets its earlier path.  The result is exactly the serial greedy parse.
+//   * Bit-pack (a4): each lane emits its path's tokens (positions combined in
+//     32-bit pairs), a 64-lane scan of bit counts places them, edge words are
+//     OR-ed, and the payload goes to the chunk's bucket with 16-byte stores.
+//   * params.version = 2 replaces the build and walk by the paper's V2 search
+//     (every position, every offset, warp argmax); chunks of S = 64..2048 are
+//     packed 4096 / S to a pair (PACK).
 
 #include "culzss_internal.h"
 
