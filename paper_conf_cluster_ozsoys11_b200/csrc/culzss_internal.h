@@ -37,7 +37,7 @@ inline void set_packing(Geometry *g) {
     g->smask = pack ? S - 1 : 4095;
 }
 
-// Per-warp shared memory.  Per-position arrays use a SKEWED layout: 4 pad
+// Per-chunk (warp pair) shared memory.  Per-position arrays use a SKEWED layout: 4 pad
 // bytes after every 128-position segment, so that the 32 lanes (one segment
 // each) scanning the same relative offset hit 32 different banks.  The pad
 // word of a segment duplicates the first word of the next one, so an
@@ -58,7 +58,7 @@ struct __align__(16) WarpSmem {
         uint8_t link[kSkewBytes];                    // distance to previous same-hash position
         union {
             uint16_t tab[(1 << kHashBits) * 32];     // [hash][lane]: u16 position + 0x1000 (W > 128)
-                                                     // or u8 position mod 256, 512 buckets (W <= 128)
+                                                     // or [lane][bucket] u8 position mod 256, 512 buckets (W <= 128)
             struct {
                 uint8_t pad[kStagePad];              // staging = link + pad (after the walks)
                 uint32_t xfer[8];                    // cross-warp exchange (exits, flags, bit counts)
