@@ -298,6 +298,8 @@ def main():
         out_n = r
         step_ms.append(ms)
     torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
     launches = culzss.launch_count() - launches0
     clk = clocks.stop()
     # per-kernel device times (roofline of the chunk kernel): the same call with
