@@ -419,9 +419,19 @@ def main():
                 dms.append(culzss.last_kernel_ms("decode"))
                 cms.append(ev0.elapsed_time(ev1))
         ok = bool(torch.equal(dec, x))
+        # decoder roofline: HBM-bound at (r + 1) bytes per output
+        # byte -- the stream read once, the output written once -- over the
+        # device time of the walk + decode kernels
+        dk = statistics.mean(dms)
+        dec_bytes = out_n + n
         line["decompress"] = {"value": n / (statistics.mean(cms) / 1000) / 1e9, "unit": "GB/s (output)",
-                              "decode_kernel_ms": statistics.mean(dms), "call_ms": statistics.mean(cms),
-                              "roundtrip_exact": ok}
+                              "decode_kernel_ms": dk, "call_ms": statistics.mean(cms),
+                              "roundtrip_exact": ok,
+                              "roofline": {"bound": "hbm", "kernels": "walk_kernel + decode_kernel",
+                                           "algorithmic_bytes": dec_bytes,
+                                           "achieved": dec_bytes / (dk / 1000) / 1e9, "peak": hbm_peak,
+                                           "unit": "GB/s", "frac": dec_bytes / (dk / 1000) / 1e9 / hbm_peak,
+                                           "peak_kind": peak_kind}}
         del dec
 
     # NEXT-1 sharded decompression at N > 1: every rank decodes its own chunk
