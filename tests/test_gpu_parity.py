@@ -382,3 +382,45 @@ def test_packed_small_chunks_match_and_tokens(env, S):
             np.testing.assert_array_equal(D[c * S:c * S + chunk.size], eD, err_msg=f"v{version} c{c}")
             np.testing.assert_array_equal(tok[c * S:c * S + chunk.size],
                                           expand_tokens(O.tokens_chunk(chunk), chunk.size))
+
+
+@pytest.mark.parametrize("S,version", [(256, 0), (4096, 2), (512, 2), (1000, 0)])
+def test_host_api_param_combinations(env, S, version):
+    """The pipelined host path (several 8 MiB groups) with packed small chunks
+    and with version 2: the same bytes as the oracle."""
+    torch, culzss = env
+    n = 2 * (8 << 20) + 4097
+    x = datagen.generate("tarmix", n, seed=S + version)
+    p = culzss.Params.make(S=S, version=version)
+    h = culzss.compress_host(x, params=p).tobytes()
+    C = (n + S - 1) // S
+    sizes = np.frombuffer(h[32:32 + 4 * C], "<u4").astype(np.int64)
+    offs = np.concatenate([[0], np.cumsum(sizes)]) + 32 + 4 * C
+    assert offs[-1] == len(h)
+    for c in sorted({0, C - 1} | set(range(0, C, max(1, C // 40)))):
+        assert h[offs[c]:offs[c + 1]] == O.compress_chunk(x[c * S:min(n, (c + 1) * S)]), c
+
+
+@pytest.mark.parametrize("S", [64, 512, 2048])
+def test_sharded_packed_chunks_roundtrip(env, S):
+    """Sharding primitives with packed small chunks: per-rank compress_chunks
+    outputs assemble into the oracle's stream and decode back per rank."""
+    torch, culzss = env
+    n = 40 * 4096 + 3 * S + 5
+    x_np = datagen.generate("csource", n, seed=S)
+    x = dev(torch, x_np)
+    p = culzss.Params.make(S=S)
+    C = (n + S - 1) // S
+    parts, tables = [], []
+    for r in range(3):
+        c0, c1 = r * C // 3, (r + 1) * C // 3
+        sl = x[c0 * S:min(c1 * S, n)]
+        pay = torch.empty(max(1, culzss.max_compressed_size(sl.numel(), p)), dtype=torch.uint8, device="cuda")
+        sizes = torch.zeros(max(1, c1 - c0), dtype=torch.int32, device="cuda")
+        t = culzss.compress_chunks(sl, pay, sizes, p)
+        assert torch.equal(culzss.decompress_chunks(pay[:t], sizes[:c1 - c0], sl.numel(), params=p), sl)
+        parts.append(pay[:t].cpu().numpy().tobytes())
+        tables.append(sizes[:c1 - c0].cpu().numpy().astype("<u4").tobytes())
+    ref = O.compress(x_np, S=S)
+    assert ref[32:32 + 4 * C] == b"".join(tables)
+    assert ref[32 + 4 * C:] == b"".join(parts)
