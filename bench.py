@@ -169,9 +169,26 @@ def cpu_baseline(x: np.ndarray, stream_bytes: bytes | None, budget_s: float = 10
         start = 32 + 4 * Ctot
         parity = bool(np.array_equal(sizes, gpu_sizes)
                       and stream_bytes[start:start + len(payload)] == payload)
+    # single-core figure beside the all-core one: one thread
+    # over a ~1 s sample of the same leading chunks
+    n1 = int(max(1, min(nchunks, 1.0 / max(per_chunk, 1e-6))))
+    t0 = time.perf_counter()
+    oracle.compress_range(x, 0, n1)
+    dt1 = time.perf_counter() - t0
+    cpu_model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                cpu_model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
     return {"value": nbytes / dt / 1e9, "unit": UNIT, "cores": len(bounds), "kind": "oracle",
             "sample": f"first {nchunks} chunks ({nbytes} B) of the same input, {len(bounds)} threads "
                       f"over contiguous chunk ranges, {dt:.2f} s wall",
+            "single_core": {"value": min(x.size, n1 * S) / dt1 / 1e9, "unit": UNIT,
+                            "sample": f"first {n1} chunks, 1 thread, {dt1:.2f} s"},
+            "cpu_model": cpu_model,
             "parity_with_gpu_stream": parity}
 
 
