@@ -281,6 +281,7 @@ def main():
     # the per-kernel split comes from separate profiled calls after the timed region
     culzss.set_profiling(True, call_only=True)
     placed = [None]
+    exch_ms = []  # N > 1: device time of the all-gather of totals per step
 
     def step():
         if world == 1:
@@ -295,6 +296,7 @@ def main():
         ev1.record(stream)
         ev1.synchronize()
         placed[0] = sharding.placements(tot, n * world, S)[rank]
+        exch_ms.append(ev0.elapsed_time(ev1))
         return t, ms_lib + ev0.elapsed_time(ev1)
 
     for _ in range(args.warmup):
@@ -390,6 +392,11 @@ def main():
         "clocks": clk,
         "gpu_launches": launches,
     }
+    if world > 1:
+        # the one exchange step: its share of a step
+        ex = statistics.mean(exch_ms[args.warmup:args.warmup + args.steps]) if exch_ms else None
+        line["exchange"] = {"op": f"{backend} all_gather_into_tensor of int64 per-rank totals",
+                            "ms_per_step": ex, "share_of_step": ex / ms_per_step if ex else None}
     # params.version = 2 (the paper's V2 search design: every position, every
     # window offset) on the same input, same protocol, fewer
     # steps: the measured cost of the brute-force design the default replaces
