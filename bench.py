@@ -508,7 +508,7 @@ def main():
         line["e2e"] = {"value": n_total / (e2e_ms / 1000) / 1e9, "unit": UNIT,
                        "h2d_bytes_per_step": n, "d2h_bytes_per_step": int(on),
                        "api": "culzss_compress_host (pinned host in/out)"}
-    if rank == 0 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:  # the CPU baseline at N = 1 only
         sb = out[:out_n].cpu().numpy().tobytes() if world == 1 else None
         line["cpu_baseline"] = cpu_baseline(x_np, sb)
     if world > 1:
