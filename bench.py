@@ -508,6 +508,25 @@ def main():
         line["e2e"] = {"value": n_total / (e2e_ms / 1000) / 1e9, "unit": UNIT,
                        "h2d_bytes_per_step": n, "d2h_bytes_per_step": int(on),
                        "api": "culzss_compress_host (pinned host in/out)"}
+        if world == 1 and "decompress" in line:
+            # host-to-host decompression of the same stream (culzss_decompress_host)
+            hdec = torch.empty(n, dtype=torch.uint8).pin_memory()
+            dtimes = []
+            for it in range(args.warmup + max(3, args.steps // 2)):
+                ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                torch.cuda.synchronize()
+                ev0.record(stream)
+                culzss.decompress_host_ptr(hout.data_ptr(), int(on), hdec.data_ptr(), n)
+                ev1.record(stream)
+                ev1.synchronize()
+                if it >= args.warmup:
+                    dtimes.append(ev0.elapsed_time(ev1))
+            line["decompress"]["e2e"] = {"value": n / (statistics.mean(dtimes) / 1000) / 1e9,
+                                         "unit": "GB/s (output)", "h2d_bytes_per_step": int(on),
+                                         "d2h_bytes_per_step": n,
+                                         "roundtrip_exact": bool(torch.equal(hdec, hin)),
+                                         "api": "culzss_decompress_host (pinned host in/out)"}
+            del hdec
     if rank == 0 and world == 1 and not args.no_cpu_baseline:  # the CPU baseline at N = 1 only
         sb = out[:out_n].cpu().numpy().tobytes() if world == 1 else None
         line["cpu_baseline"] = cpu_baseline(x_np, sb)

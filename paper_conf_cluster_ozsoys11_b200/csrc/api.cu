@@ -554,14 +554,8 @@ culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host
     return CULZSS_OK;
 }
 
-static culzss_status read_header(const void *in, size_t in_n, Geometry *g, uint64_t *n,
-                                 uint64_t *C, cudaStream_t st) {
-    if (in_n < 32) return CULZSS_ERR_CORRUPT;
-    uint64_t *hw = host_word();
-    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
-    uint8_t *h = reinterpret_cast<uint8_t *>(hw);
-    CK(cudaMemcpyAsync(h, in, 32, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
+// Parse and validate the 32-byte header from host bytes (readings R12, R13).
+static culzss_status parse_header(const uint8_t *h, Geometry *g, uint64_t *n, uint64_t *C) {
     auto le = [&](int off, int nb) {
         uint64_t v = 0;
         for (int i = 0; i < nb; i++) v |= (uint64_t)h[off + i] << (8 * i);
@@ -586,6 +580,17 @@ static culzss_status read_header(const void *in, size_t in_n, Geometry *g, uint6
     return s == CULZSS_OK ? CULZSS_OK : CULZSS_ERR_UNSUPPORTED;
 }
 
+static culzss_status read_header(const void *in, size_t in_n, Geometry *g, uint64_t *n,
+                                 uint64_t *C, cudaStream_t st) {
+    if (in_n < 32) return CULZSS_ERR_CORRUPT;
+    uint64_t *hw = host_word();
+    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
+    uint8_t *h = reinterpret_cast<uint8_t *>(hw);
+    CK(cudaMemcpyAsync(h, in, 32, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    return parse_header(h, g, n, C);
+}
+
 culzss_status culzss_decompressed_size(const void *in, size_t in_n, size_t *n,
                                        culzss_stream_t stream) {
     lib_init();
@@ -598,37 +603,48 @@ culzss_status culzss_decompressed_size(const void *in, size_t in_n, size_t *n,
     return s == CULZSS_ERR_UNSUPPORTED ? CULZSS_OK : s;
 }
 
-// Decode C chunks (n output bytes) from `payload` (pay_len bytes) with the
-// u32 size table at `table_src` (device, any alignment: copied to an aligned
-// workspace).  Scan of the sizes, walk + decode kernels, one sync for the
-// device error word.
-static culzss_status decompress_core(const uint8_t *payload, uint64_t pay_len, const void *table_src, uint64_t C,
-                                     uint64_t n, const Geometry &g, uint8_t *out, cudaStream_t st) {
-    // workspace: aligned copy of the table | offsets | scan ws | total | err
+// Enqueue the decode of C chunks (n output bytes) from `payload` (pay_len
+// bytes) with the u32 size table at `table_src` (device, any alignment:
+// copied to an aligned workspace) on st, without a host sync: scan of the
+// sizes, walk + decode kernels; malformed chunks OR bits into *err (device).
+static culzss_status decompress_enqueue(const uint8_t *payload, uint64_t pay_len, const void *table_src, uint64_t C,
+                                        uint64_t n, const Geometry &g, uint8_t *out, cudaStream_t st, uint32_t *err,
+                                        bool prof) {
+    // workspace: aligned copy of the table | offsets | scan ws | total | records
     const uint64_t tab_off = 0;
     const uint64_t offs_off = (C * 4 + 255) / 256 * 256;
     const uint64_t ws_off = offs_off + (C * 8 + 255) / 256 * 256;
     const uint64_t tot_off = ws_off + (scan_workspace_words(C) * 8 + 255) / 256 * 256;
     const uint64_t tb_off = tot_off + 256;
-    Workspace ws(st);
+    Workspace ws(st);  // freed stream-ordered on st
     CK(ws.alloc(tb_off + decode_scratch_bytes(C)));
     uint8_t *base = static_cast<uint8_t *>(ws.p);
     uint32_t *sizes = reinterpret_cast<uint32_t *>(base + tab_off);
     uint64_t *offsets = reinterpret_cast<uint64_t *>(base + offs_off);
     uint64_t *scanws = reinterpret_cast<uint64_t *>(base + ws_off);
     uint64_t *total = reinterpret_cast<uint64_t *>(base + tot_off);
-    uint32_t *err = reinterpret_cast<uint32_t *>(base + tot_off + 8);
     CK(cudaMemcpyAsync(sizes, table_src, C * 4, cudaMemcpyDeviceToDevice, st));
-    CK(cudaMemsetAsync(err, 0, 4, st));
     CK(launch_scan(sizes, C, offsets, total, scanws, st));
-    uint64_t *hw = host_word();
-    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
     // the walk kernel checks the table against the payload length (no sync here)
-    t_prof.reset();
-    t_prof.rec(1, st);
+    if (prof) t_prof.rec(1, st);
     CK(launch_decode(payload, pay_len, sizes, offsets, C, n, g, out, err, reinterpret_cast<uint32_t *>(base + tb_off),
                      st));
-    t_prof.rec(2, st);
+    if (prof) t_prof.rec(2, st);
+    return CULZSS_OK;
+}
+
+// Synchronous decode: enqueue, then one sync for the device error word.
+static culzss_status decompress_core(const uint8_t *payload, uint64_t pay_len, const void *table_src, uint64_t C,
+                                     uint64_t n, const Geometry &g, uint8_t *out, cudaStream_t st) {
+    Workspace ew(st);
+    CK(ew.alloc(256));
+    uint32_t *err = static_cast<uint32_t *>(ew.p);
+    CK(cudaMemsetAsync(err, 0, 4, st));
+    uint64_t *hw = host_word();
+    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
+    t_prof.reset();
+    culzss_status s = decompress_enqueue(payload, pay_len, table_src, C, n, g, out, st, err, true);
+    if (s != CULZSS_OK) return s;
     CK(cudaMemcpyAsync(hw, err, 4, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     if (t_profiling) t_times.decode = t_prof.between(1, 2);
@@ -678,6 +694,114 @@ culzss_status culzss_decompress_chunks(const void *payload, size_t payload_n, co
         return CULZSS_ERR_INVALID_ARG;
     return decompress_core(static_cast<const uint8_t *>(payload), payload_n, chunk_sizes, C, slice_n, g,
                            static_cast<uint8_t *>(out), (cudaStream_t)stream);
+}
+
+// Host-memory decompression, the inverse of culzss_compress_host: the
+// header and size table are read from host memory, the output is decoded in
+// groups of ~8 MiB on the three compute streams (H2D of the group's table
+// slice and payload, scan + walk + decode), and each group's output is copied
+// back on the copy stream as soon as its kernels finish, so both copy
+// directions overlap the kernels.  Device errors OR into one word checked at
+// the single final sync.
+culzss_status culzss_decompress_host(const void *in_host, size_t in_n, void *out_host, size_t *out_n,
+                                     const culzss_params *, culzss_stream_t stream) {
+    lib_init();
+    if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
+    if (!out_n || !in_host || !out_host) return CULZSS_ERR_INVALID_ARG;
+    if (in_n < 32) return CULZSS_ERR_CORRUPT;
+    const uint8_t *hin = static_cast<const uint8_t *>(in_host);
+    Geometry g;
+    uint64_t n, C;
+    culzss_status s = parse_header(hin, &g, &n, &C);
+    if (s != CULZSS_OK) return s;
+    if (in_n < 32 + 4 * C) return CULZSS_ERR_CORRUPT;
+    if (*out_n < n) {
+        *out_n = (size_t)n;
+        return CULZSS_ERR_BUFFER_TOO_SMALL;
+    }
+    if (n == 0) {
+        if (in_n != 32) return CULZSS_ERR_CORRUPT;
+        *out_n = 0;
+        return CULZSS_OK;
+    }
+    // payload offsets from the host copy of the table (u64 prefix sums)
+    std::vector<uint64_t> off(C + 1, 0);
+    for (uint64_t c = 0; c < C; c++) {
+        uint32_t v;
+        memcpy(&v, hin + 32 + 4 * c, 4);
+        off[c + 1] = off[c] + v;
+    }
+    const uint64_t pay_len = in_n - 32 - 4 * C;
+    if (off[C] != pay_len) return CULZSS_ERR_CORRUPT;
+    cudaStream_t st = (cudaStream_t)stream;
+    static const uint64_t dgroup_bytes = [] {  // CULZSS_DGROUP_KB: decode group size (output bytes)
+        const char *e = getenv("CULZSS_DGROUP_KB");
+        const long v = e ? atol(e) : 0;
+        return v > 0 ? (uint64_t)v << 10 : (8ull << 20);
+    }();
+    const uint64_t gc = std::max<uint64_t>(1, dgroup_bytes / g.S);  // chunks per group
+    const uint64_t G = (C + gc - 1) / gc;
+    HostPipe &hp = t_pipe;
+    if (!hp.init(G)) return cuda_fail(cudaErrorMemoryAllocation);
+    // device: table | payload | output | error word
+    const uint64_t tab_bytes = (4 * C + 255) / 256 * 256;
+    const uint64_t pay_bytes = (pay_len + 255) / 256 * 256;
+    const uint64_t out_bytes = (n + 255) / 256 * 256;
+    Workspace ws(st);
+    CK(ws.alloc(tab_bytes + pay_bytes + out_bytes + 256));
+    uint8_t *dtab = static_cast<uint8_t *>(ws.p);
+    uint8_t *dpay = dtab + tab_bytes;
+    uint8_t *dout = dpay + pay_bytes;
+    uint32_t *err = reinterpret_cast<uint32_t *>(dout + out_bytes);
+    uint8_t *hout = static_cast<uint8_t *>(out_host);
+    struct Drain {  // on an error return, no internal stream may still use ws
+        HostPipe &hp;
+        bool done = false;
+        ~Drain() {
+            if (done) return;
+            for (auto cs : hp.cs) cudaStreamSynchronize(cs);
+            cudaStreamSynchronize(hp.ds);
+            cudaGetLastError();
+        }
+    } drain{hp};
+    t_prof.reset();
+    t_prof.rec(0, st);
+    CK(cudaMemsetAsync(err, 0, 4, st));
+    CK(cudaEventRecord(hp.ev_in, st));  // the workspace exists and the error word is clear
+    for (auto cs : hp.cs) CK(cudaStreamWaitEvent(cs, hp.ev_in, 0));
+    CK(cudaStreamWaitEvent(hp.ds, hp.ev_in, 0));
+    for (uint64_t k = 0; k < G; k++) {
+        cudaStream_t cs = hp.cs[k % kPipeStreams];
+        const uint64_t c0 = k * gc, c1 = std::min(C, c0 + gc);
+        const uint64_t b0 = c0 * g.S, nb = std::min<uint64_t>(n, c1 * g.S) - b0;
+        CK(cudaMemcpyAsync(dtab + 4 * c0, hin + 32 + 4 * c0, 4 * (c1 - c0), cudaMemcpyHostToDevice, cs));
+        if (off[c1] > off[c0])
+            CK(cudaMemcpyAsync(dpay + off[c0], hin + 32 + 4 * C + off[c0], off[c1] - off[c0],
+                               cudaMemcpyHostToDevice, cs));
+        s = decompress_enqueue(dpay + off[c0], off[c1] - off[c0], dtab + 4 * c0, c1 - c0, nb, g, dout + b0, cs, err,
+                               false);
+        if (s != CULZSS_OK) return s;
+        CK(cudaEventRecord(hp.ev[k], cs));
+        CK(cudaStreamWaitEvent(hp.ds, hp.ev[k], 0));
+        CK(cudaMemcpyAsync(hout + b0, dout + b0, nb, cudaMemcpyDeviceToHost, hp.ds));
+    }
+    // the caller's stream resumes after everything (the workspace is freed on it)
+    CK(cudaEventRecord(hp.ev_in, hp.ds));
+    CK(cudaStreamWaitEvent(st, hp.ev_in, 0));
+    for (auto cs : hp.cs) {
+        CK(cudaEventRecord(hp.ev[0], cs));
+        CK(cudaStreamWaitEvent(st, hp.ev[0], 0));
+    }
+    uint64_t *hw = host_word();
+    if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
+    CK(cudaMemcpyAsync(hw, err, 4, cudaMemcpyDeviceToHost, st));
+    t_prof.rec(5, st);
+    CK(cudaStreamSynchronize(st));
+    drain.done = true;
+    if (t_profiling) t_times.call = t_prof.between(0, 5);
+    if (reinterpret_cast<uint32_t *>(hw)[0]) return CULZSS_ERR_CORRUPT;
+    *out_n = (size_t)n;
+    return CULZSS_OK;
 }
 
 static culzss_status debug_entry(int mode, const void *in, size_t n, void *dst,

@@ -8,6 +8,7 @@ there is no CPU fallback.
 from __future__ import annotations
 
 import ctypes
+import struct
 import os
 from typing import Optional, Tuple
 
@@ -67,6 +68,7 @@ def _lib():
             getattr(L, name).argtypes = [vp, sz, vp, szp, pp, vp]
         L.culzss_decompressed_size.argtypes = [vp, sz, szp, vp]
         L.culzss_decompress.argtypes = [vp, sz, vp, szp, pp, vp]
+        L.culzss_decompress_host.argtypes = [vp, sz, vp, szp, pp, vp]
         L.culzss_compress_chunks.argtypes = [vp, sz, vp, szp, vp, pp, vp]
         L.culzss_decompress_chunks.argtypes = [vp, sz, vp, sz, vp, pp, vp]
         L.culzss_write_header.argtypes = [vp, sz, pp, vp]
@@ -199,6 +201,35 @@ def decompress_status(s, out=None, stream=None) -> Tuple[int, object]:
     st = _lib().culzss_decompress(ctypes.c_void_p(s.data_ptr()), s.numel(), ctypes.c_void_p(out.data_ptr()),
                                   ctypes.byref(on), None, _stream(stream))
     return st, (out[: on.value] if st == OK else None)
+
+
+def decompress_host_status(s: np.ndarray, out: Optional[np.ndarray] = None, stream=None) -> Tuple[int, object]:
+    """Host-memory decompression (H2D + decode + D2H pipelined inside the library)."""
+    s = np.ascontiguousarray(s, dtype=np.uint8)
+    if out is None:
+        n = struct.unpack_from("<Q", s.tobytes()[16:24])[0] if s.size >= 32 else 0
+        if n > 122 * s.size + 1:  # memory guard: a valid stream expands < 122x
+            return ERR_CORRUPT, None
+        out = np.empty(max(n, 1), dtype=np.uint8)
+    on = ctypes.c_size_t(out.size)
+    st = _lib().culzss_decompress_host(ctypes.c_void_p(s.ctypes.data), s.size, ctypes.c_void_p(out.ctypes.data),
+                                       ctypes.byref(on), None, _stream(stream))
+    return st, (out[: on.value] if st == OK else None)
+
+
+def decompress_host(s: np.ndarray, out: Optional[np.ndarray] = None, stream=None) -> np.ndarray:
+    st, o = decompress_host_status(s, out, stream)
+    _check(st, "culzss_decompress_host")
+    return o
+
+
+def decompress_host_ptr(in_ptr: int, in_n: int, out_ptr: int, cap: int, stream=None) -> int:
+    """culzss_decompress_host on raw host pointers (e.g. pinned torch tensors)."""
+    on = ctypes.c_size_t(cap)
+    st = _lib().culzss_decompress_host(ctypes.c_void_p(in_ptr), in_n, ctypes.c_void_p(out_ptr), ctypes.byref(on),
+                                       None, _stream(stream))
+    _check(st, "culzss_decompress_host")
+    return on.value
 
 
 def decompress(s, out=None, stream=None):

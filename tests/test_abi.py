@@ -30,7 +30,7 @@ def test_header_declares_expected_entry_points():
     for s in ("culzss_compress", "culzss_decompress", "culzss_compress_chunks", "culzss_write_header",
               "culzss_max_compressed_size", "culzss_default_params", "culzss_status_string",
               "culzss_match_search", "culzss_parse_tokens", "culzss_compress_host",
-              "culzss_decompress_chunks"):
+              "culzss_decompress_chunks", "culzss_decompress_host"):
         assert s in syms
 
 

@@ -424,3 +424,49 @@ def test_sharded_packed_chunks_roundtrip(env, S):
     ref = O.compress(x_np, S=S)
     assert ref[32:32 + 4 * C] == b"".join(tables)
     assert ref[32 + 4 * C:] == b"".join(parts)
+
+
+@pytest.mark.parametrize("kind,n,S", [("csource", (8 << 20) + 1, 4096), ("tarmix", 3 * (8 << 20) + 4097 * 3 + 17, 4096),
+                                      ("random", 2 * (8 << 20), 4096), ("runs20", 5 * (8 << 20) - 1, 4096),
+                                      ("english", 100_001, 4096), ("csource", 3 * (8 << 20) + 5, 512),
+                                      ("english", 1, 4096)])
+def test_decompress_host(env, kind, n, S):
+    """Host-memory decompression of oracle streams (single and multi-group,
+    packed chunk size), byte-exact."""
+    torch, culzss = env
+    x = datagen.generate(kind, n, seed=n % 1000)
+    # small inputs: the oracle's stream; large: the GPU stream (whose chunks the
+    # oracle checks in the other tests) -- the host decoder must return the input
+    s = np.frombuffer(O.compress(x, S=S), np.uint8) if n < (1 << 20) else \
+        culzss.compress_host(x, params=culzss.Params.make(S=S))
+    y = culzss.decompress_host(s)
+    assert y.tobytes() == x.tobytes()
+    # pinned buffers through the raw-pointer entry point
+    sin = torch.from_numpy(np.array(s, dtype=np.uint8)).pin_memory()
+    out = torch.empty(n + 7, dtype=torch.uint8).pin_memory()
+    on = culzss.decompress_host_ptr(sin.data_ptr(), s.size, out.data_ptr() + 3, n + 4)
+    assert on == n and out[3:3 + n].numpy().tobytes() == x.tobytes()
+
+
+def test_decompress_host_rejects(env):
+    torch, culzss = env
+    import test_oracle_pins as P
+    for _, s in P.CORRUPT_STREAMS:
+        st, _ = culzss.decompress_host_status(np.frombuffer(s, np.uint8))
+        assert st == culzss.ERR_CORRUPT, s
+    x = datagen.generate("english", 20000, seed=4)
+    base = bytearray(O.compress(x))
+    rng = np.random.default_rng(7)
+    for _ in range(100):
+        s = bytearray(base)
+        for _ in range(int(rng.integers(1, 4))):
+            i = int(rng.integers(0, len(s)))
+            s[i] ^= int(rng.integers(1, 256))
+        ost, oout = O.decompress_status(bytes(s))
+        gst, gout = culzss.decompress_host_status(np.frombuffer(bytes(s), np.uint8))
+        if ost == O.OK:
+            assert gst == culzss.OK and gout.tobytes() == oout
+        else:
+            assert gst in (culzss.ERR_CORRUPT, culzss.ERR_UNSUPPORTED)
+    st, _ = culzss.decompress_host_status(np.frombuffer(bytes(base), np.uint8), out=np.empty(10, np.uint8))
+    assert st == culzss.ERR_BUFFER_TOO_SMALL
