@@ -55,6 +55,9 @@ def parse_args():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-decompress", action="store_true")
+    ap.add_argument("--assemble", action="store_true",
+                    help="N > 1: also gather the whole stream on rank 0 (point-to-point sends of every "
+                         "rank's table slice and payload; timed separately, not part of the metric)")
     ap.add_argument("--no-versions", action="store_true",
                     help="skip timing params.version = 2 (the paper's V2 all-position search) beside the default")
     return ap.parse_args()
@@ -281,6 +284,7 @@ def main():
     # the per-kernel split comes from separate profiled calls after the timed region
     culzss.set_profiling(True, call_only=True)
     placed = [None]
+    last_totals = [None]
     exch_ms = []  # N > 1: device time of the all-gather of totals per step
 
     def step():
@@ -296,6 +300,7 @@ def main():
         ev1.record(stream)
         ev1.synchronize()
         placed[0] = sharding.placements(tot, n * world, S)[rank]
+        last_totals[0] = tot
         exch_ms.append(ev0.elapsed_time(ev1))
         return t, ms_lib + ev0.elapsed_time(ev1)
 
@@ -392,6 +397,31 @@ def main():
         "clocks": clk,
         "gpu_launches": launches,
     }
+    if world > 1 and args.assemble:
+        # optional assembly on rank 0, verified by a
+        # device round trip against every rank's (regenerated) input
+        tpay = culzss.compress_chunks(x, payload, sizes)
+        pay_t, sz_t = payload[:tpay], sizes[:C]
+        if backend != "nccl":
+            pay_t, sz_t = pay_t.cpu(), sz_t.cpu()
+        torch.cuda.synchronize()
+        dist.barrier()
+        t0 = time.perf_counter()
+        full = sharding.assemble_on_root_tensors(pay_t, sz_t, last_totals[0], n * world, (S, 128, 128, 3))
+        torch.cuda.synchronize()
+        dist.barrier()
+        wall = (time.perf_counter() - t0) * 1000
+        if rank == 0:
+            full = full.to(dev)
+            y = culzss.decompress(full)
+            ok = all(torch.equal(y[r * n:(r + 1) * n].cpu(), torch.from_numpy(rank_input(args.config, r, world)))
+                     for r in range(world))
+            line["assembly"] = {"wall_ms": wall, "stream_bytes": int(full.numel()),
+                                "gbps_into_rank0": full.numel() / (wall / 1000) / 1e9,
+                                "op": f"{backend} point-to-point sends of table slices and payloads to rank 0",
+                                "roundtrip_exact": bool(ok)}
+            del y
+        del full
     if world > 1:
         # the one exchange step: its share of a step
         ex = statistics.mean(exch_ms[args.warmup:args.warmup + args.steps]) if exch_ms else None

@@ -142,3 +142,50 @@ def assemble_on_root(payload: bytes, sizes_le: bytes, place: RankPlacement, n_to
         pos += len(pay)
     assert pos == place.stream_bytes
     return bytes(buf)
+
+
+def assemble_on_root_tensors(payload, sizes, totals: Sequence[int], n_total: int,
+                             params: Tuple[int, int, int, int], group=None):
+    """Assembly with point-to-point transfers of tensors:
+    every rank sends its u32 size-table slice and its payload straight into
+    their final byte ranges of rank 0's output tensor (NCCL send/recv over
+    NVLink for CUDA tensors; gloo for CPU tensors).  `payload` is this rank's
+    uint8 payload (exactly its total), `sizes` its int32 table slice,
+    `totals` the all-gathered per-rank totals.  Returns the stream tensor on
+    rank 0, None elsewhere."""
+    import torch
+    import torch.distributed as dist
+    rank = dist.get_rank(group)
+    world = dist.get_world_size(group)
+    S, W, F, MIN = params
+    pl = placements(totals, n_total, S)
+    me = pl[rank]
+    tab = (sizes.contiguous().view(torch.uint8) if sizes.numel()
+           else torch.empty(0, dtype=torch.uint8, device=sizes.device))
+    if rank != 0:
+        reqs = []
+        if me.c1 > me.c0:
+            reqs.append(dist.isend(tab, dst=0, group=group))
+        if me.payload_bytes:
+            reqs.append(dist.isend(payload.contiguous(), dst=0, group=group))
+        for r in reqs:
+            r.wait()
+        return None
+    out = torch.empty(me.stream_bytes, dtype=torch.uint8, device=payload.device)
+    out[:HEADER_BYTES] = torch.frombuffer(bytearray(header(n_total, S, W, F, MIN)), dtype=torch.uint8).to(out.device)
+    reqs = []
+    for p in pl:
+        tsl = out[p.table_offset:p.table_offset + 4 * (p.c1 - p.c0)]
+        psl = out[p.payload_offset:p.payload_offset + p.payload_bytes]
+        if p.rank == 0:
+            tsl.copy_(tab)
+            psl.copy_(payload)
+            continue
+        if p.c1 > p.c0:
+            reqs.append(dist.irecv(tsl, src=p.rank, group=group))
+        if p.payload_bytes:
+            reqs.append(dist.irecv(psl, src=p.rank, group=group))
+    for r in reqs:
+        r.wait()
+    return out
+

@@ -137,3 +137,48 @@ def test_stream_views_closed_form():
     assert all(p.stream_bytes == 32 + 4 * C + sum(sizes) for p in v)
     with pytest.raises(ValueError):
         sharding.stream_views(sizes[:-1], n, S, 2)
+
+
+def _asm_worker(rank, world, port, kind, n, S, out_q):
+    """Tensor assembly on rank 0 through point-to-point transfers (gloo here;
+    NCCL send/recv on B200s)."""
+    import torch
+    import torch.distributed as dist
+    import oracle as O
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        x = datagen.generate(kind, n, seed=31)
+        C = sharding.n_chunks(n, S)
+        c0, c1 = sharding.chunk_range(rank, world, C)
+        if c1 > c0:
+            pay, sizes = O.compress_range(x, c0, c1, S=S)
+        else:
+            pay, sizes = b"", np.zeros(0, np.uint32)
+        pay_t = torch.frombuffer(bytearray(pay), dtype=torch.uint8) if pay else torch.empty(0, dtype=torch.uint8)
+        sizes_t = torch.from_numpy(np.asarray(sizes, dtype=np.uint32).view(np.int32).copy())
+        totals = sharding.exchange_totals(len(pay))
+        out = sharding.assemble_on_root_tensors(pay_t, sizes_t, totals, n, (S, 128, 128, 3))
+        if rank == 0:
+            out_q.put(out.numpy().tobytes())
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,kind,n,S", [(2, "csource", 37 * 4096 + 1111, 4096),
+                                            (3, "tarmix", 5000, 1000),
+                                            (4, "random", 2 * 4096, 4096)])  # ranks with no chunks
+def test_tensor_assembly_gloo(world, kind, n, S):
+    import oracle as O
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_asm_worker, args=(r, world, port, kind, n, S, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert out == O.compress(datagen.generate(kind, n, seed=31), S=S)
