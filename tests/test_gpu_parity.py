@@ -470,3 +470,26 @@ def test_decompress_host_rejects(env):
             assert gst in (culzss.ERR_CORRUPT, culzss.ERR_UNSUPPORTED)
     st, _ = culzss.decompress_host_status(np.frombuffer(bytes(base), np.uint8), out=np.empty(10, np.uint8))
     assert st == culzss.ERR_BUFFER_TOO_SMALL
+
+
+@pytest.mark.parametrize("cfg", ["c2_csource_128m", "c3_runs20_1g", "c4_random_1g"])
+def test_full_size_configs_every_chunk(env, cfg):
+    """BASELINE configs at full size: EVERY chunk of the GPU stream against the
+    oracle (threads over contiguous chunk ranges on the box's host cores), plus
+    the header and the size table."""
+    import concurrent.futures as cf
+    import os
+    torch, culzss = env
+    spec = datagen.CONFIGS[cfg]
+    x_np = datagen.generate(spec["kind"], spec["n"], spec["seed"])
+    stream = culzss.compress(torch.from_numpy(x_np).cuda()).cpu().numpy().tobytes()
+    n, S = x_np.size, 4096
+    C = (n + S - 1) // S
+    assert stream[:32] == struct.pack("<4sHHIIQHHB3x", b"CLZS", 1, 32, S, C, n, 128, 128, 3)
+    k = max(1, min(len(os.sched_getaffinity(0)), 64))
+    bounds = [(i * C // k, (i + 1) * C // k) for i in range(k)]
+    with cf.ThreadPoolExecutor(k) as ex:
+        res = list(ex.map(lambda b: O.compress_range(x_np, b[0], b[1]), bounds))
+    sizes = np.concatenate([r[1] for r in res]).astype("<u4").tobytes()
+    assert stream[32:32 + 4 * C] == sizes
+    assert stream[32 + 4 * C:] == b"".join(r[0] for r in res)
