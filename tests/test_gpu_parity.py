@@ -472,7 +472,7 @@ def test_decompress_host_rejects(env):
     assert st == culzss.ERR_BUFFER_TOO_SMALL
 
 
-@pytest.mark.parametrize("cfg", ["c2_csource_128m", "c3_runs20_1g", "c4_random_1g"])
+@pytest.mark.parametrize("cfg", ["c2_csource_128m", "c3_runs20_1g", "c4_random_1g", "c5_tarmix_1g_slice"])
 def test_full_size_configs_every_chunk(env, cfg):
     """BASELINE configs at full size: EVERY chunk of the GPU stream against the
     oracle (threads over contiguous chunk ranges on the box's host cores), plus
@@ -480,7 +480,10 @@ def test_full_size_configs_every_chunk(env, cfg):
     import concurrent.futures as cf
     import os
     torch, culzss = env
-    spec = datagen.CONFIGS[cfg]
+    if cfg == "c5_tarmix_1g_slice":  # 1 GiB of the c5 generator (its per-rank slices are 8 GiB at dp8)
+        spec = dict(datagen.CONFIGS["c5_tarmix_64g"], n=1 << 30)
+    else:
+        spec = datagen.CONFIGS[cfg]
     x_np = datagen.generate(spec["kind"], spec["n"], spec["seed"])
     stream = culzss.compress(torch.from_numpy(x_np).cuda()).cpu().numpy().tobytes()
     n, S = x_np.size, 4096
