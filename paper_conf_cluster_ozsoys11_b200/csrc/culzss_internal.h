@@ -13,11 +13,11 @@ constexpr int kChunkMax = 4096;     // largest chunk the kernel stages (S <= 409
 constexpr int kSeg = 128;           // positions per lane segment (32 x 128 = 4096)
 constexpr int kHashBits = 8;        // per-lane 3-gram hash table, W > 128: 256 u16 heads
 constexpr int kHashBitsSmallW = 9;  // W <= 128: 512 u8 heads (relative positions)
-constexpr int kChunksPerCta = 3;    // chunks per CTA
+constexpr int kChunksPerCta = 1;    // chunks per CTA (each chunk's smem is released when it finishes)
 constexpr int kWarpsPerChunk = 2;   // warp 0 builds the hash chains; all warps walk
 constexpr int kWalkLanes = 32 * kWarpsPerChunk;   // 64 walk segments per chunk
 constexpr int kWSeg = kChunkMax / kWalkLanes;     // 64 positions per walk segment
-constexpr int kCtasPerSm = 3;
+constexpr int kCtasPerSm = 9;
 
 struct Geometry {
     uint32_t S, W, F;               // chunk, window, max match (MIN is 3)
@@ -53,7 +53,8 @@ constexpr int kStageWords = ((kWSeg * 9 + 17 + 31) / 32) | 1;   // odd stride: c
 constexpr int kStagePad = (kWalkLanes * kStageWords * 4 > kSkewBytes ? kWalkLanes * kStageWords * 4 - kSkewBytes : 0) + 16;
 constexpr int kUcwWords = kChunkMax / 4 + 4;  // + zero tail: 8-byte loads read 3 words
 struct __align__(16) WarpSmem {
-    uint32_t cw[(kSkewBytes + 16) / 4];              // chunk bytes (skewed) + zero tail
+    uint32_t cw[kSkewBytes / 4];                     // chunk bytes (skewed).  No tail: reads past the
+                                                     // chunk end only feed bytes beyond every match's cap
     struct {
         uint8_t link[kSkewBytes];                    // distance to previous same-hash position
         union {

@@ -332,17 +332,15 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     uint8_t *link = sm.a.link;
 
     // ---------------- a1: stage the chunk (16-byte coalesced loads) --------
-    // a full chunk overwrites every data byte: only the zero tail (read by
-    // the 8-byte compares past the end) needs clearing, and no barrier has to
-    // order the clearing before the data stores
+    // a full chunk overwrites every data byte, so nothing needs clearing and
+    // no barrier has to order the clearing before the data stores (bytes past
+    // the chunk end are only ever read beyond a match's cap)
     const bool full = m == kChunkMax;
     {
         uint4 *z4 = reinterpret_cast<uint4 *>(sm.cw);
         const uint4 z = make_uint4(0, 0, 0, 0);
         if (!full) {
             for (int i = t64; i < (int)(sizeof(sm.cw) / 16); i += kWalkLanes) z4[i] = z;
-        } else if (t64 == 0) {
-            z4[sizeof(sm.cw) / 16 - 1] = z;
         }
         uint4 *t4 = reinterpret_cast<uint4 *>(sm.a.u.tab);
         // u8 tables: empty = (s0 - 129) mod 256 = 0x7F (even lanes) / 0xFF (odd)
@@ -487,7 +485,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
 #pragma unroll 4
         for (int i = t64; i < (int)(sizeof(sm.a.u.w.ld) / 16); i += kWalkLanes) l4[i] = z;
 #pragma unroll 4
-        for (int j = t64; j < kUcwWords; j += kWalkLanes) ucw[j] = __byte_perm(sm.cw[j + (j >> 5)], 0, 0x0123);
+        for (int j = t64; j < kUcwWords; j += kWalkLanes)
+            ucw[j] = j < kChunkMax / 4 ? __byte_perm(sm.cw[j + (j >> 5)], 0, 0x0123) : 0u;  // + zero tail
     }
     // candidate mask: bit i = position s0 + i (< s1) has a chain link
     uint32_t rc0 = 0, rc1 = 0;
