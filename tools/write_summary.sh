@@ -38,7 +38,7 @@ echo
 echo "### Per-phase split of the c2 chunk kernel (tools/ncu_lines.py: warp instructions / warp stall samples by source line range)"
 echo
 echo '```'
-python tools/ncu_lines.py gpurun_out/full_c2_csource_128m_$TAG.ncu-rep lzss_chunk.cu ${RANGES:-56:142:helpers 143:242:walk 243:323:v2 324:359:stage 360:438:build 439:485:mask 486:527:fixup 528:598:emit 599:670:scan+write} --top 15
+python tools/ncu_lines.py gpurun_out/full_c2_csource_128m_$TAG.ncu-rep lzss_chunk.cu ${RANGES:-56:138:helpers 139:244:walk 245:306:v2 307:376:stage 377:473:build 474:515:mask 516:569:fixup 570:648:emit 649:736:scan+write} --top 15
 echo '```'
 echo
 echo "## Decoder (row a6), --set full, c2 stream"
