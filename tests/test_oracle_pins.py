@@ -236,6 +236,26 @@ CORRUPT_STREAMS = [
     ("reserved", _stream(1, lit("a"))[:29] + b"\x01\x00\x00" + _stream(1, lit("a"))[32:]),
     ("bad params", struct.pack("<4sHHIIQHHB3x", b"CLZS", 1, 32, 4096, 1, 1, 0, 128, 3)
      + struct.pack("<I", 2) + bits_to_bytes(lit("a"))),
+    # Each stream below is valid in every respect but ONE, so each isolates
+    # one rejection branch of the decoder (DESIGN.md §3 decoder strictness;
+    # PAPER.md:1@6743 §II.A.2 decode rule; readings R9, R10, R12).
+    # d = 5 > W = 4, though d <= produced (5) and L = 3 <= remaining (3)
+    ("d > W", header(8, W=4) + struct.pack("<I", len(bits_to_bytes("".join(lit(ch) for ch in "abcde") + mat(5, 3))))
+     + bits_to_bytes("".join(lit(ch) for ch in "abcde") + mat(5, 3))),
+    # L = 6 > F = 5, though L <= remaining (6) and d = 1 <= produced
+    ("L > F", header(7, F=5) + struct.pack("<I", len(bits_to_bytes(lit("a") + mat(1, 6))))
+     + bits_to_bytes(lit("a") + mat(1, 6))),
+    # header version 2 (R12 fixes version = 1)
+    ("version", _stream(1, lit("a"))[:4] + struct.pack("<H", 2) + _stream(1, lit("a"))[6:]),
+    # header_bytes = 64 (R12 fixes 32)
+    ("header_bytes", _stream(1, lit("a"))[:6] + struct.pack("<H", 64) + _stream(1, lit("a"))[8:]),
+    # C = 1 < ceil(4097 / 4096) = 2, with a table and payload that agree with
+    # C = 1 (the one chunk decodes 4096 bytes cleanly): only the C check sees it
+    ("C too small", struct.pack("<4sHHIIQHHB3x", b"CLZS", 1, 32, 4096, 1, 4097, 128, 128, 3)
+     + struct.pack("<I", len(bits_to_bytes(lit("z") + mat(1, 128) * 31 + mat(1, 127))))
+     + bits_to_bytes(lit("z") + mat(1, 128) * 31 + mat(1, 127))),
+    # C = 0 for n = 1: an empty table and no payload
+    ("C zero", struct.pack("<4sHHIIQHHB3x", b"CLZS", 1, 32, 4096, 0, 1, 128, 128, 3)),
 ]
 
 
@@ -243,6 +263,21 @@ CORRUPT_STREAMS = [
 def test_decoder_rejects_corrupt(name, stream):
     st, _ = O.decompress_status(stream)
     assert st == O.ERR_CORRUPT, name
+
+
+def test_isolating_streams_decode_once_fixed():
+    """Positive controls for the isolating corrupt streams: with the one bad
+    field set right, each decodes (so the rejection above is that field's)."""
+    five = "".join(lit(ch) for ch in "abcde")
+    ok_w = header(8, W=5) + struct.pack("<I", len(bits_to_bytes(five + mat(5, 3)))) + bits_to_bytes(five + mat(5, 3))
+    assert O.decompress(ok_w) == b"abcdeabc"
+    ok_f = header(7, F=6) + struct.pack("<I", len(bits_to_bytes(lit("a") + mat(1, 6)))) + bits_to_bytes(lit("a") + mat(1, 6))
+    assert O.decompress(ok_f) == b"a" * 7
+    pay = bits_to_bytes(lit("z") + mat(1, 128) * 31 + mat(1, 127))
+    ok_c = (struct.pack("<4sHHIIQHHB3x", b"CLZS", 1, 32, 4096, 1, 4096, 128, 128, 3)
+            + struct.pack("<I", len(pay)) + pay)
+    assert O.decompress(ok_c) == b"z" * 4096
+    assert O.decompress(_stream(1, lit("a"))) == b"a"
 
 
 def test_params_validation():
