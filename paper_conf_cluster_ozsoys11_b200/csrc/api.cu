@@ -81,6 +81,8 @@ culzss_status check_params(const culzss_params *p, Geometry *g) {
     if ((p->version != 0 && p->version != 2) || p->chunk_size > (uint32_t)kChunkMax || p->window > 255)
         return CULZSS_ERR_UNSUPPORTED;
     g->V = p->version;
+    if (const char *e = getenv("CULZSS_WALK_SWITCH")) g->sw = (uint32_t)atol(e);
+    if (const char *e = getenv("CULZSS_WALK_TOKEN_SWITCH")) g->tx = (uint32_t)atol(e);
     g->S = p->chunk_size;
     g->W = p->window;
     g->F = p->max_match;
@@ -167,7 +169,19 @@ struct Prof {
         for (auto &u : used) u = false;
     }
 };
-thread_local Prof t_prof;
+// CUDA events and streams belong to the device that was current when they
+// were created: the per-thread state is kept per device ordinal.
+constexpr int kMaxDevices = 64;
+int cur_device() {
+    int d = 0;
+    if (cudaGetDevice(&d) != cudaSuccess) {
+        cudaGetLastError();
+        d = 0;
+    }
+    return d >= 0 && d < kMaxDevices ? d : 0;
+}
+thread_local Prof t_prof_dev[kMaxDevices];
+#define t_prof (t_prof_dev[cur_device()])
 
 void prof_finish_compress() {
     if (!t_profiling) return;
@@ -366,7 +380,11 @@ culzss_status culzss_compress_chunks(const void *in_slice, size_t slice_n, void 
         *payload_n = 0;
         return CULZSS_OK;
     }
+    if (n_chunks(slice_n, g.S) > 0xFFFFFFFFull) return CULZSS_ERR_INVALID_ARG;
     if (!is_device_ptr(in_slice) || !is_device_ptr(payload) || !is_device_ptr(chunk_sizes))
+        return CULZSS_ERR_INVALID_ARG;
+    if (overlap(in_slice, slice_n, payload, bound) || overlap(in_slice, slice_n, chunk_sizes, 4 * n_chunks(slice_n, g.S)) ||
+        overlap(payload, bound, chunk_sizes, 4 * n_chunks(slice_n, g.S)))
         return CULZSS_ERR_INVALID_ARG;
     uint64_t *hw = host_word();
     if (!hw) return cuda_fail(cudaErrorMemoryAllocation);
@@ -387,6 +405,37 @@ culzss_status culzss_compress_chunks(const void *in_slice, size_t slice_n, void 
     prof_finish_compress();
     *payload_n = (size_t)*hw;
     return CULZSS_OK;
+}
+
+culzss_status culzss_compress_chunks_async(const void *in_slice, size_t slice_n, void *payload,
+                                           size_t payload_cap, uint32_t *chunk_sizes, uint64_t *dev_total,
+                                           const culzss_params *p, culzss_stream_t stream) {
+    lib_init();
+    if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
+    Geometry g;
+    culzss_status s = check_params(p, &g);
+    if (s != CULZSS_OK) return s;
+    const uint64_t bound = payload_bound(slice_n, g.S);
+    if (payload_cap < bound) return CULZSS_ERR_BUFFER_TOO_SMALL;
+    const uint64_t C = n_chunks(slice_n, g.S);
+    if (C > 0xFFFFFFFFull) return CULZSS_ERR_INVALID_ARG;
+    if (!is_device_ptr(dev_total) || (reinterpret_cast<uintptr_t>(dev_total) & 7)) return CULZSS_ERR_INVALID_ARG;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (slice_n == 0) {
+        CK(cudaMemsetAsync(dev_total, 0, 8, st));
+        return CULZSS_OK;
+    }
+    if (!is_device_ptr(in_slice) || !is_device_ptr(payload) || !is_device_ptr(chunk_sizes))
+        return CULZSS_ERR_INVALID_ARG;
+    if (overlap(in_slice, slice_n, payload, bound) || overlap(in_slice, slice_n, chunk_sizes, 4 * C) ||
+        overlap(payload, bound, chunk_sizes, 4 * C) || overlap(dev_total, 8, payload, bound) ||
+        overlap(dev_total, 8, chunk_sizes, 4 * C) || overlap(dev_total, 8, in_slice, slice_n))
+        return CULZSS_ERR_INVALID_ARG;
+    const CoreLayout lay(C, g.S);
+    Workspace ws(st);  // freed stream-ordered on st after the kernels
+    CK(ws.alloc(lay.total));
+    return compress_core(static_cast<const uint8_t *>(in_slice), slice_n, g, static_cast<uint8_t *>(payload),
+                         nullptr, chunk_sizes, dev_total, st, ws.p, false);
 }
 
 // Pipelined host-memory compression: the chunks go in groups of ~8 MiB.
@@ -431,7 +480,7 @@ struct HostPipe {
         return true;
     }
 };
-thread_local HostPipe t_pipe;
+thread_local HostPipe t_pipe_dev[kMaxDevices];  // streams/events of the current device
 }  // namespace
 
 culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host, size_t *out_n,
@@ -472,7 +521,7 @@ culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host
         *out_n = on;
         return CULZSS_OK;
     }
-    HostPipe &hp = t_pipe;
+    HostPipe &hp = t_pipe_dev[cur_device()];
     if (!hp.init(G)) return cuda_fail(cudaErrorMemoryAllocation);
     // device: input | header + table (contiguous, as in the stream) | per-group
     // staging at its worst-case offset | group totals | two core workspaces
@@ -741,7 +790,7 @@ culzss_status culzss_decompress_host(const void *in_host, size_t in_n, void *out
     }();
     const uint64_t gc = std::max<uint64_t>(1, dgroup_bytes / g.S);  // chunks per group
     const uint64_t G = (C + gc - 1) / gc;
-    HostPipe &hp = t_pipe;
+    HostPipe &hp = t_pipe_dev[cur_device()];
     if (!hp.init(G)) return cuda_fail(cudaErrorMemoryAllocation);
     // device: table | payload | output | error word
     const uint64_t tab_bytes = (4 * C + 255) / 256 * 256;

@@ -2,6 +2,7 @@
 // Not part of the ABI (the ABI is include/culzss.h).  Shares nothing with
 // oracle/ (independence rule).
 #pragma once
+#include <atomic>
 #include <cstddef>
 #include <cstdint>
 #include <cuda_runtime.h>
@@ -26,6 +27,12 @@ struct Geometry {
     uint32_t K = 1;                 // chunks per warp pair: 4096 / S for S in {64, 128, ..., 2048},
                                     // else 1 (small chunks packed into one 4096-position buffer)
     uint32_t smask = 4095;          // S - 1 when K > 1: position p's chunk is [p & ~smask, +S)
+    uint32_t tx = 16;               // iterations one lane may spend on one token before its warp
+                                    // switches to the pruned walk machine (B200 sweep:
+                                    // profiles/r2_walk_switch.md), ...
+    uint32_t sw = 1u << 30;         // ... or walk iterations of the warp in total (off by default).
+                                    // CULZSS_WALK_TOKEN_SWITCH / CULZSS_WALK_SWITCH override both, for
+                                    // tuning and for the tests that cover each machine on its own
 };
 // Chunk packing for the fused kernel: chunks of S = 64 .. 2048
 // (powers of two) share one warp pair, K = 4096 / S of them, so every 64-position
@@ -71,6 +78,7 @@ struct __align__(16) WarpSmem {
     } a;
 };
 static_assert(sizeof(WarpSmem) <= 24848, "smem layout");
+static_assert(kChunkMax / 32 * 4 <= kStagePad, "run-boundary mask (one bit per position) fits in the staging pad");
 static_assert(offsetof(WarpSmem, a.u.w.xfer) - offsetof(WarpSmem, a.link) >= kWalkLanes * kStageWords * 4,
               "staging (over link + pad) must not reach xfer / ld");
 static_assert((kChunkMax * 9 / 8 + 16) <= sizeof(WarpSmem::a.u.w.ld), "payload words fit in ld");
@@ -96,6 +104,21 @@ cudaError_t launch_decode(const uint8_t *payload, uint64_t pay_len, const uint32
 uint64_t decode_scratch_bytes(uint64_t C);
 
 void count_launch(int k = 1);
+
+// cudaFuncSetAttribute opt-ins (dynamic shared memory above 48 KB) apply to
+// the CURRENT device only: done once per (kernel, device), tracked in a
+// per-kernel bit mask of device ordinals.
+template <typename K>
+cudaError_t set_smem_attr_once(K kernel, int bytes, std::atomic<uint64_t> &done) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    const uint64_t bit = dev < 64 ? 1ull << dev : 0;
+    if (bit && (done.load(std::memory_order_relaxed) & bit)) return cudaSuccess;
+    e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes);
+    if (e == cudaSuccess && bit) done.fetch_or(bit, std::memory_order_relaxed);
+    return e;
+}
 
 }  // namespace culzss
 

@@ -105,35 +105,174 @@ __device__ __forceinline__ uint32_t hash9(uint32_t w) { return (w * kHashMul) >>
 
 __device__ __forceinline__ int tok_len(uint32_t t) { return t >= 0x100 ? (int)(t & 0xFF) + 3 : 1; }
 
-// Token at one position by a plain chain walk (debug entry point only).
-__device__ uint32_t eval_pos(const uint32_t *cw, const uint8_t *link, int p, int m, int W, int F) {
+// Run-boundary mask (the run-skip prune): bit x of bnd (u32
+// words, position-indexed) = chunk[x] != chunk[x+1]; every bit from the
+// chunk's last position on is set.  run_len / run_start read it with ffs /
+// clz (a run of equal bytes of length up to 128 spans at most 5 words).
+//
+// length of the run of equal bytes starting at p, capped at cap (>= 1)
+__device__ __forceinline__ int run_len(const uint32_t *__restrict__ bnd, int p, int cap) {
+    int x = p;
+    uint32_t w = bnd[x >> 5] >> (x & 31);
+    int r = 0;
+    while (!w) {  // no boundary in the rest of this word
+        r += 32 - (x & 31);
+        if (r >= cap) return cap;
+        x = (x | 31) + 1;
+        w = bnd[x >> 5];
+    }
+    return min(r + __ffs(w), cap);
+}
+// first position of the run of equal bytes that contains q, or lo if that
+// run starts at or before lo (lo < q)
+__device__ __forceinline__ int run_start(const uint32_t *__restrict__ bnd, int q, int lo) {
+    int x = q - 1;  // the run starts after the last boundary bit below q
+    while (x >= lo) {
+        const uint32_t w = bnd[x >> 5] << (31 - (x & 31));  // bit 31 = position x
+        if (w) return max(x - (int)__clz(w) + 1, lo);
+        x = (x & ~31) - 1;
+    }
+    return lo;
+}
+
+// The same two run queries read on the fly from the big-endian chunk copy u
+// (for eval_pos: a fix-up re-walk may run in a warp without the mask).
+__device__ __forceinline__ int run_len_u(const uint32_t *__restrict__ u, int p, int cap) {
+    const Be8 f = load8(u, p);
+    const uint64_t B = (uint64_t)(f.hi >> 24) * 0x0101010101010101ull;
+    uint64_t v = (((uint64_t)f.hi << 32) | f.lo) ^ B;
+    int k = 0;
+    while (!v) {
+        k += 8;
+        if (k >= cap) return cap;
+        const Be8 w = load8(u, p + k);
+        v = (((uint64_t)w.hi << 32) | w.lo) ^ B;
+    }
+    return min(k + (__clzll(v) >> 3), cap);
+}
+__device__ __forceinline__ int run_start_u(const uint32_t *__restrict__ u, int q, int lo) {
+    const Be8 f = load8(u, q);
+    const uint64_t B = (uint64_t)(f.hi >> 24) * 0x0101010101010101ull;
+    int x = q;  // the run covers [x, q]
+    while (x > lo) {
+        const int a = max(x - 8, lo);  // bytes [a, x): the first x - a of the 8 loaded
+        const Be8 w = load8(u, a);
+        const uint64_t v = ((((uint64_t)w.hi << 32) | w.lo) ^ B) >> (8 * (8 - (x - a)));
+        if (v) return x - (__ffsll(v) - 1) / 8;  // equal bytes just below x
+        x = a;
+    }
+    return lo;
+}
+
+// Longest common prefix of the chunk at q and at p (q < p), capped at cap,
+// 8 bytes per step on the big-endian copy u.
+__device__ __forceinline__ int lcp8(const uint32_t *__restrict__ u, int q, int p, int cap) {
+    int k = 0;
+    while (k < cap) {
+        const Be8 a = load8(u, q + k), b = load8(u, p + k);
+        const int fb = __clzll(((uint64_t)(a.hi ^ b.hi) << 32) | (a.lo ^ b.lo)) >> 3;
+        k += fb;
+        if (fb < 8) break;
+    }
+    return min(k, cap);
+}
+
+// first entry > dmin of the chain through position z (link hops, chain
+// offset already applied), starting from distance d0 = that of z; 0 if the
+// chain ends or passes wlim first
+__device__ __forceinline__ int chain_after(const uint8_t *__restrict__ link, int p, int o, int d0, int dmin,
+                                           int wlim) {
+    int d = d0;
+    while (d <= dmin) {
+        const int l2 = link[sk(p - d + o)];
+        if (!l2) return 0;
+        d += l2;
+    }
+    return d <= wlim ? d : 0;
+}
+
+// (L, D) at one position p by the chain walk with the same two exact prunes
+// as the walk state machine below (a plain loop: fix-up re-walks only).
+// m: end of p's chunk, cstart: its start.  Returns the memo encoding.
+__device__ uint32_t eval_pos(const uint32_t *__restrict__ u, const uint8_t *__restrict__ link, int p, int m,
+                             int cstart, int W, int F) {
     const int cap = min(F, m - p);
-    if (cap < 3) return kLit;
     int d = link[sk(p)];
-    int bestL = 2, bestD = 0;
+    if (cap < 3 || !d) return kLit;
+    const int wlim = min(W, p - cstart);
+    int t = -1;  // run length at p (computed when first needed)
+    int bestL = 2, bestD = 0, o = 0, nrej = 0;
     while (d) {
         const int q = p - d;
-        int k = 0;
-        while (true) {
-            const uint32_t x = load4(cw, q + k) ^ load4(cw, p + k);
-            if (x) {
-                k += (__ffs(x) - 1) >> 3;
-                break;
-            }
-            k += 4;
-            if (k >= cap) break;
-        }
-        const int L = min(k, cap);
-        if (L > bestL) {
+        const int L = lcp8(u, q, p, cap);
+        const bool upd = L > bestL;
+        if (upd) {
             bestL = L;
             bestD = d;
             if (L == cap) break;
         }
-        const int l2 = link[sk(q)];
-        if (!l2 || d + l2 > W) break;
-        d += l2;
+        nrej = upd ? 0 : nrej + 1;
+        if (L >= 3 && t < 0) t = run_len_u(u, p, cap);
+        if (L >= 3 && L < t) {
+            // run skip: q's match ended with the run of equal bytes it sits in
+            const int lo = p - wlim;
+            const int r0 = run_start_u(u, q, lo);
+            const int qs = max(q + L - t, r0);
+            if (qs < q) {
+                const int L2 = lcp8(u, qs, p, cap);
+                if (L2 > bestL) {
+                    bestL = L2;
+                    bestD = p - qs;
+                    if (L2 == cap) break;
+                }
+                if (r0 <= lo) break;
+                o = 0;  // resume on p's own chain after the run start
+                nrej = 0;
+                d = chain_after(link, p, 0, p - r0, p - r0, wlim);
+                continue;
+            }
+        }
+        if (nrej >= 2 && bestL >= 3 && bestL - 2 > o) {
+            // chain switch: every better candidate matches bytes [bestL-2, bestL]
+            o = bestL - 2;
+            nrej = 0;
+            const int e = link[sk(p + o)];
+            d = e ? chain_after(link, p, o, e, d, wlim) : 0;
+            continue;
+        }
+        const int l2 = link[sk(q + o)];
+        d = (l2 && d + l2 <= wlim) ? d + l2 : 0;
     }
     return bestD ? ((uint32_t)bestD << 8) | (uint32_t)(bestL - 3) : kLit;
+}
+
+// Run-boundary mask of a warp's half of the chunk plus the 5 words each side
+// that run_len / run_start reach from it (positions [2048h - 160, 2048h +
+// 2208)), built on demand by the whole warp when it switches to the pruned
+// walk.  Both warps of a pair may write the shared words in between, with
+// identical values.  The skewed words of one 32-position group lie in one
+// 128-position segment; the group's next word is the pad word (a copy of the
+// next segment's first word) at a segment end.
+__device__ __forceinline__ void build_bnd_warp(const uint32_t *__restrict__ cw, uint32_t *__restrict__ bnd,
+                                               int half, int lane, int m) {
+    const int w0 = max(64 * half - 5, 0), w1 = min(64 * half + 69, kChunkMax / 32);
+#pragma unroll 1
+    for (int w = w0 + lane; w < w1; w += 32) {
+        const uint32_t *c = cw + (sk(32 * w) >> 2);
+        uint32_t a = c[0], bits = 0;
+#pragma unroll
+        for (int gi = 0; gi < 8; gi++) {
+            const uint32_t an = c[gi + 1];
+            const uint32_t v = a ^ __funnelshift_r(a, an, 8);  // byte j: chunk[x+j] ^ chunk[x+j+1]
+            const uint32_t nz = (((v & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | v) & 0x80808080u;
+            bits |= ((nz >> 7) * 0x10204080u >> 28) << (4 * gi);  // bit j = byte j nonzero
+            a = an;
+        }
+        const int lim = m - 1 - 32 * w;  // bits from the last position m-1 on are set
+        if (lim < 32) bits |= lim <= 0 ? 0xFFFFFFFFu : ~((1u << lim) - 1);
+        bnd[w] = bits;
+    }
+    __syncwarp();
 }
 
 // Speculative greedy walk over segment [s0, s1) from s0 as a branch-free
@@ -149,11 +288,32 @@ __device__ uint32_t eval_pos(const uint32_t *cw, const uint8_t *link, int p, int
 //   * a finished token is memoised in ld[] and p jumps over candidate-free
 //     positions (literals) with the lane's candidate mask; the new token's
 //     first candidate is loaded in the same iteration.
+// A warp still walking after `sw` iterations, or one of whose lanes has spent
+// `tx` iterations on one token (runs and structured binary: long chains of
+// true 3-gram candidates), continues in a second machine with
+// two exact prunes, after building its run-boundary mask;
+// there a finished candidate moves to the next one on the chain it was found
+// on (d += link[p-d+o]) or, in a rarely taken branch:
+//   - run skip: a candidate whose match L (3 <= L < t, t = the run of equal
+//     bytes at p) ended because the run it sits in ended: the start
+//     qs = max(end - t, run start) of that run dominates every other start in
+//     it (nearer ones match less, farther ones at most as much), so qs is
+//     evaluated next and the walk then resumes after the run start on p's
+//     chain;
+//   - chain switch: after two candidates in a row that did not improve,
+//     continue on the chain of p's 3-gram at offset o = bestL-2 (any better
+//     candidate matches those bytes too), from its first entry beyond d.
+// Both keep the candidates in increasing d, so the strict '>' still leaves
+// the smallest d on ties (reading R7).
+// ALLPOS (per-position parity dump, row a2): every candidate position of the
+// segment is evaluated and (L, D) written to dump instead.
 // Returns the exit (first position >= s1 the greedy path reaches).
+template <bool ALLPOS>
 __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const uint8_t *__restrict__ link,
-                                         uint64_t cm, uint16_t *__restrict__ ld, int m, int W,
-                                         int F, int s0,
-                                         int s1, bool &anym) {
+                                         const uint32_t *__restrict__ cw, uint32_t *__restrict__ bnd, uint64_t cm,
+                                         uint16_t *__restrict__ ld, uint8_t *__restrict__ dump, int m, int mbuf,
+                                         int cstart, int W, int F, int s0, int s1, int half, int lane, int sw,
+                                         int tx, bool &anym) {
     // token starts stay inside the lane's segment, which never crosses a
     // 128-position skew boundary: p-indexed arrays use a constant offset
     const int so = (s0 >> 7) << 2;
@@ -169,8 +329,31 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
     }
     int k = 0, bestL = 2, bestD = 0;
     int qr = 0;  // reject-test mode (int: no byte-register repacking)
+    auto finish_token = [&]() {
+        if (ALLPOS) {
+            dump[2 * p] = (uint8_t)(bestD ? bestL : 0);
+            dump[2 * p + 1] = (uint8_t)bestD;
+        } else {
+            lds[p] = (uint16_t)(bestD ? (bestD << 8) | (bestL - 3) : kLit);
+        }
+        nm |= bestD;
+        p = next_cand(cm, p + (ALLPOS ? 1 : (bestD ? bestL : 1)), s0, s1);
+        active = p < s1;
+        if (active) {
+            d = lks[p];
+            cap = min(F, m - p);
+        }
+        bestL = 2;
+        bestD = 0;
+        k = 0;
+        qr = 0;
+    };
+    // ---- machine 1: plain chain walk, until the warp has walked sw
+    // iterations or one of its lanes has spent tx on its current token ------
+    int it = 0, ti = 0;  // warp iterations, iterations of the lane's current token
 #pragma unroll 1
-    while (__any_sync(kFull, active)) {
+    for (; it < sw && __any_sync(kFull, active) && !__any_sync(kFull, active && ti >= tx); it++) {
+        ti++;
         if (active) {
             const int q = p - d;
             const int off = qr ? bestL - 7 : k;
@@ -200,18 +383,84 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
                 qr = bestL >= 8 ? 1 : 0;
             }
             if (tok_done) {
-                lds[p] = (uint16_t)(bestD ? (bestD << 8) | (bestL - 3) : kLit);
-                nm |= bestD;
-                p = next_cand(cm, p + (bestD ? bestL : 1), s0, s1);
-                active = p < s1;
-                if (active) {
-                    d = lks[p];
-                    cap = min(F, m - p);
+                finish_token();
+                ti = 0;
+            }
+        }
+    }
+    if (__any_sync(kFull, active)) {
+        // ---- machine 2: the same walk with the two exact prunes ------------
+        build_bnd_warp(cw, bnd, half, lane, mbuf);
+        const int wl0 = min(W, p - cstart);
+        int wlim = wl0;          // window limit of p: min(W, p - chunk start)
+        int o = 0;               // chain offset (chain switch)
+        int rs = 0;              // run skip: distance of the run start to resume after (0: none; > W: stop)
+        int nrej = 0;            // candidates since the last improvement
+        bool runp = false;       // bytes p..p+3 are equal (latched when off == 0)
+#pragma unroll 1
+        while (__any_sync(kFull, active)) {
+            if (active) {
+                const int q = p - d;
+                const int off = qr ? bestL - 7 : k;
+                int lq;
+                asm volatile("ld.volatile.shared.u8 %0, [%1];"
+                             : "=r"(lq)
+                             : "r"((uint32_t)__cvta_generic_to_shared(link + sk(q + o))));
+                const Be8 vq = load8(u, q + off), vp = load8(u, p + off);
+                const uint32_t xh = vq.hi ^ vp.hi, xl = vq.lo ^ vp.lo;
+                const int fb = __clzll(((uint64_t)xh << 32) | xl) >> 3;
+                runp = off == 0 ? vp.hi == __byte_perm(vp.hi, 0, 0x3333) : runp;
+                const bool cand_done = fb < 8 || (!qr && k + 8 >= cap);
+                const int L = min(k + fb, cap);
+                const bool lval = !qr && cand_done;  // L is the finished candidate's match length
+                const bool upd = lval && L > bestL;
+                bestL = upd ? L : bestL;
+                bestD = upd ? d : bestD;
+                k = qr ? 0 : k + 8;
+                qr = qr && fb < 8 ? 1 : 0;
+                bool tok_done = false;
+                if (cand_done) {
+                    nrej = upd ? 0 : nrej + 1;
+                    int nd = d + lq;
+                    bool fin = lq == 0 || nd > wlim || bestL == cap;  // default: follow the chain
+                    if (!fin || rs) {
+                        if (rs) {  // qs done: resume after the run start on p's own chain
+                            nd = rs <= wlim ? chain_after(link, p, 0, rs, rs, wlim) : 0;
+                            fin = nd == 0 || bestL == cap;
+                            o = 0;
+                            rs = 0;
+                            nrej = 0;
+                        } else if (lval && runp && L >= 3) {
+                            const int t = run_len(bnd, p, cap);
+                            if (L < t) {
+                                const int lo = p - wlim;
+                                const int r0 = run_start(bnd, q, lo);
+                                const int qs = max(q + L - t, r0);
+                                if (qs < q) {  // run skip (else q starts its run: follow the chain)
+                                    nd = p - qs;
+                                    rs = r0 > lo ? p - r0 : 0x7FFF;
+                                }
+                            }
+                        } else if (nrej >= 2 && bestL >= 3 && bestL - 2 > o) {  // chain switch
+                            o = bestL - 2;
+                            nrej = 0;
+                            const int e = link[sk(p + o)];
+                            nd = e ? chain_after(link, p, o, e, d, wlim) : 0;
+                            fin = nd == 0;
+                        }
+                    }
+                    d = nd;
+                    tok_done = fin;
+                    k = 0;
+                    qr = bestL >= 8 ? 1 : 0;
                 }
-                bestL = 2;
-                bestD = 0;
-                k = 0;
-                qr = 0;
+                if (tok_done) {
+                    finish_token();
+                    wlim = min(W, p - cstart);
+                    o = 0;
+                    rs = 0;
+                    nrej = 0;
+                }
             }
         }
     }
@@ -225,8 +474,8 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
 // there is the same.  A later re-walk of the same lane (rare: its entry moved
 // twice) cannot tell which earlier walk a memoised start belongs to and walks
 // to the segment end, reusing memoised tokens.
-__device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restrict__ link, uint64_t cm,
-                        uint16_t *__restrict__ ld, int m, int W, int F, int s0, int s1, int entry,
+__device__ int walk_fix(const uint32_t *__restrict__ u, const uint8_t *__restrict__ link, uint64_t cm,
+                        uint16_t *__restrict__ ld, int m, int cstart, int W, int F, int s0, int s1, int entry,
                         int spec_exit, bool first) {
     int p = entry;
     while (true) {
@@ -235,7 +484,7 @@ __device__ int walk_fix(const uint32_t *__restrict__ cw, const uint8_t *__restri
         uint32_t t = ld[sk2(p)];
         if (t && first) return spec_exit;
         if (!t) {
-            t = eval_pos(cw, link, p, m, W, F);
+            t = eval_pos(u, link, p, m, cstart, W, F);
             ld[sk2(p)] = (uint16_t)t;
         }
         p += tok_len(t);
@@ -459,12 +708,11 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         pair_sync(bar);
     }
 
-    if (MODE == kModeDumpMatch) {
-        // every position, for per-position parity (a2)
+    if (V2 && MODE == kModeDumpMatch) {
+        // every position's evaluated token, for per-position parity (a2)
         uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
         for (int p = t64; p < m; p += kWalkLanes) {
-            const uint32_t t = V2 ? (uint32_t)sm.a.u.w.ld[sk2(p)]
-                                  : eval_pos(sm.cw, link, p, min((p | smask) + 1, m), W, F);
+            const uint32_t t = sm.a.u.w.ld[sk2(p)];
             LD[2 * p] = (uint8_t)(t == kLit ? 0 : (t & 0xFF) + 3);
             LD[2 * p + 1] = (uint8_t)(t == kLit ? 0 : t >> 8);
         }
@@ -475,8 +723,10 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     const int s0 = t64 * kWSeg;
     const int s1 = min(s0 + kWSeg, m);  // <= s0 for lanes past the chunk end
     const int ce = PACK ? min((s0 | smask) + 1, m) : m;  // end of the segment's chunk (matches stop there)
+    const int cst = PACK ? (s0 & ~smask) : 0;  // start of the segment's chunk
     uint16_t *ld = sm.a.u.w.ld;
     uint32_t *ucw = sm.a.u.w.ucw;
+    uint32_t *bnd = reinterpret_cast<uint32_t *>(sm.a.u.w.pad);  // free until the bit-pack staging
     if (!V2) {
         // zero the memoised tokens (their bytes held the hash tables) and
         // unskew the chunk for the walks' compares
@@ -515,7 +765,16 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     pair_sync(bar);
     bool anym = true;  // the speculative path holds a match (V2: not tracked)
     const uint64_t cm = ((uint64_t)rc0 << 32) | rc1;
-    const int spec_exit = V2 ? v2_jump(ld, s0, s1) : walk_spec(ucw, link, cm, ld, ce, W, F, s0, s1, anym);
+    if (MODE == kModeDumpMatch) {
+        // every candidate position through the production walk machine (a2)
+        uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
+        walk_spec<true>(ucw, link, sm.cw, bnd, cm, ld, LD, ce, m, cst, W, F, s0, s1, half, lane, (int)g.sw,
+                        (int)g.tx, anym);
+        return;
+    }
+    const int spec_exit =
+        V2 ? v2_jump(ld, s0, s1) : walk_spec<false>(ucw, link, sm.cw, bnd, cm, ld, nullptr, ce, m, cst, W, F, s0, s1, half, lane,
+                                     (int)g.sw, (int)g.tx, anym);
     int exitp = spec_exit;
     int cur = s0;
     bool first = true;
@@ -543,7 +802,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         par ^= 1;
         if (chg) {
             exitp = V2 ? v2_jump(ld, entry, s1)
-                       : walk_fix(sm.cw, link, cm, ld, ce, W, F, s0, s1, entry, spec_exit, first);
+                       : walk_fix(ucw, link, cm, ld, ce, cst, W, F, s0, s1, entry, spec_exit, first);
             first = false;
             cur = entry;
         }
@@ -740,13 +999,9 @@ cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *buck
     const uint64_t C = (n + g.S - 1) / g.S;
     if (C == 0) return cudaSuccess;
     const size_t smem = sizeof(WarpSmem) * kChunksPerCta;
-    static bool attr_set = false;  // benign race: idempotent
-    if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(chunk_kernel<MODE, SMALLW, V2, PACK>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        attr_set = true;
-    }
+    static std::atomic<uint64_t> attr_devs{0};  // per device (the opt-in is per device context)
+    cudaError_t e = set_smem_attr_once(chunk_kernel<MODE, SMALLW, V2, PACK>, (int)smem, attr_devs);
+    if (e != cudaSuccess) return e;
     const uint64_t pairs = (C + g.K - 1) / g.K;
     const uint64_t blocks = (pairs + kChunksPerCta - 1) / kChunksPerCta;
     chunk_kernel<MODE, SMALLW, V2, PACK><<<(unsigned)blocks, kChunksPerCta * kWalkLanes, smem, st>>>(in, n, g, bucket,

@@ -22,7 +22,7 @@ OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_BUFFER_TOO_SMALL, ERR_CORRUPT, ERR_CUD
 EXPORTS = (
     "culzss_default_params", "culzss_max_compressed_size", "culzss_compress",
     "culzss_compress_host", "culzss_decompressed_size", "culzss_decompress",
-    "culzss_compress_chunks", "culzss_write_header", "culzss_match_search",
+    "culzss_compress_chunks", "culzss_compress_chunks_async", "culzss_write_header", "culzss_match_search",
     "culzss_parse_tokens", "culzss_device_count", "culzss_launch_count",
     "culzss_set_profiling", "culzss_last_kernel_ms", "culzss_status_string",
     "culzss_last_cuda_error",
@@ -70,6 +70,7 @@ def _lib():
         L.culzss_decompress.argtypes = [vp, sz, vp, szp, pp, vp]
         L.culzss_decompress_host.argtypes = [vp, sz, vp, szp, pp, vp]
         L.culzss_compress_chunks.argtypes = [vp, sz, vp, szp, vp, pp, vp]
+        L.culzss_compress_chunks_async.argtypes = [vp, sz, vp, sz, vp, vp, pp, vp]
         L.culzss_decompress_chunks.argtypes = [vp, sz, vp, sz, vp, pp, vp]
         L.culzss_write_header.argtypes = [vp, sz, pp, vp]
         L.culzss_match_search.argtypes = [vp, sz, vp, pp, vp]
@@ -238,6 +239,15 @@ def decompress(s, out=None, stream=None):
     return o
 
 
+def _check_table_len(chunk_sizes, slice_n: int, params) -> None:
+    """The kernels write / read ceil(slice_n / S) entries of chunk_sizes: a
+    shorter tensor would be an out-of-bounds device access."""
+    S = params.chunk_size if params is not None else 4096
+    need = (slice_n + S - 1) // S if S else 0
+    if chunk_sizes.numel() < need or not chunk_sizes.is_contiguous():
+        raise ValueError(f"chunk_sizes must be a contiguous tensor of >= ceil(slice_n/S) = {need} entries")
+
+
 def compress_chunks(x_slice, payload, chunk_sizes, params: Optional[Params] = None, stream=None) -> int:
     """Sharding primitive: payload only (no header/table); returns payload bytes."""
     import torch
@@ -245,6 +255,7 @@ def compress_chunks(x_slice, payload, chunk_sizes, params: Optional[Params] = No
     _dev_u8(payload)
     if not (chunk_sizes.is_cuda and chunk_sizes.dtype == torch.int32):
         raise TypeError("chunk_sizes must be a CUDA int32 tensor (u32 bit pattern)")
+    _check_table_len(chunk_sizes, x_slice.numel(), params)
     pn = ctypes.c_size_t(payload.numel())
     st = _lib().culzss_compress_chunks(ctypes.c_void_p(x_slice.data_ptr()), x_slice.numel(),
                                        ctypes.c_void_p(payload.data_ptr()), ctypes.byref(pn),
@@ -252,6 +263,25 @@ def compress_chunks(x_slice, payload, chunk_sizes, params: Optional[Params] = No
                                        _stream(stream))
     _check(st, "culzss_compress_chunks")
     return pn.value
+
+
+def compress_chunks_async(x_slice, payload, chunk_sizes, dev_total, params: Optional[Params] = None,
+                          stream=None) -> None:
+    """Sharding primitive without a host sync: the payload total goes to the
+    CUDA int64 tensor dev_total[0] (stream-ordered) for a device all-gather."""
+    import torch
+    _dev_u8(x_slice)
+    _dev_u8(payload)
+    if not (chunk_sizes.is_cuda and chunk_sizes.dtype == torch.int32):
+        raise TypeError("chunk_sizes must be a CUDA int32 tensor (u32 bit pattern)")
+    if not (dev_total.is_cuda and dev_total.dtype == torch.int64 and dev_total.numel() >= 1):
+        raise TypeError("dev_total must be a CUDA int64 tensor")
+    _check_table_len(chunk_sizes, x_slice.numel(), params)
+    _check(_lib().culzss_compress_chunks_async(ctypes.c_void_p(x_slice.data_ptr()), x_slice.numel(),
+                                               ctypes.c_void_p(payload.data_ptr()), payload.numel(),
+                                               ctypes.c_void_p(chunk_sizes.data_ptr()),
+                                               ctypes.c_void_p(dev_total.data_ptr()), _params(params),
+                                               _stream(stream)), "culzss_compress_chunks_async")
 
 
 def decompress_chunks_status(payload, chunk_sizes, slice_n: int, out=None, params: Optional[Params] = None,
@@ -263,6 +293,7 @@ def decompress_chunks_status(payload, chunk_sizes, slice_n: int, out=None, param
     _dev_u8(payload)
     if not (chunk_sizes.is_cuda and chunk_sizes.dtype == torch.int32):
         raise TypeError("chunk_sizes must be a CUDA int32 tensor (u32 bit pattern)")
+    _check_table_len(chunk_sizes, slice_n, params)
     if out is None:
         out = torch.empty(max(slice_n, 1), dtype=torch.uint8, device=payload.device)
     _dev_u8(out)

@@ -340,17 +340,34 @@ _BASES = {"english": _english_base, "wordlist": _wordlist_base, "csource": _csou
 _BASE_CAP = {"english": 4 << 20, "wordlist": 4 << 20, "csource": 16 << 20, "tarmix": 64 << 20}
 
 
-def _tile_segments(base: np.ndarray, n: int, seed: int, seg_lo: int = 1 << 16,
-                   seg_hi: int = 1 << 20) -> np.ndarray:
+def _segment_plan(base_size: int, n: int, seed: int, seg_lo: int = 1 << 16,
+                  seg_hi: int = 1 << 20) -> list:
+    """[(pos, off, ln)]: output bytes [pos, pos + ln) = base[off:off + ln]."""
     rng = np.random.Generator(np.random.PCG64(seed ^ 0x5EED))
-    out = np.empty(n, dtype=np.uint8)
+    plan = []
     pos = 0
     while pos < n:
-        ln = min(int(rng.integers(seg_lo, seg_hi + 1)), n - pos, base.size)
-        off = int(rng.integers(0, base.size - ln + 1))
-        out[pos:pos + ln] = base[off:off + ln]
+        ln = min(int(rng.integers(seg_lo, seg_hi + 1)), n - pos, base_size)
+        off = int(rng.integers(0, base_size - ln + 1))
+        plan.append((pos, off, ln))
         pos += ln
+    return plan
+
+
+def _tile_segments(base: np.ndarray, n: int, seed: int) -> np.ndarray:
+    out = np.empty(n, dtype=np.uint8)
+    for pos, off, ln in _segment_plan(base.size, n, seed):
+        out[pos:pos + ln] = base[off:off + ln]
     return out
+
+
+def _clip_plan(plan, b0: int, b1: int):
+    """The plan's pieces that fall in [b0, b1), as (dst, src_off, ln) with dst
+    relative to b0."""
+    for pos, off, ln in plan:
+        lo, hi = max(pos, b0), min(pos + ln, b1)
+        if lo < hi:
+            yield lo - b0, off + (lo - pos), hi - lo
 
 
 def generate(kind: str, n: int, seed: int = 1) -> np.ndarray:
@@ -370,6 +387,53 @@ def generate(kind: str, n: int, seed: int = 1) -> np.ndarray:
     if n <= cap:
         return base[:n].copy()
     return _tile_segments(base, n, seed)
+
+
+def generate_range(kind: str, n: int, seed: int, b0: int, b1: int) -> np.ndarray:
+    """Bytes [b0, b1) of generate(kind, n, seed) without materialising the rest
+    where the generator allows it (random: counter-based; tiled corpora: only
+    the segments that overlap the range)."""
+    if not 0 <= b0 <= b1 <= n:
+        raise ValueError("need 0 <= b0 <= b1 <= n")
+    if kind == "random":
+        w0 = b0 // 8
+        with np.errstate(over="ignore"):
+            idx = np.arange(w0 + 1, (b1 + 7) // 8 + 1, dtype=np.uint64)
+            z = np.uint64(seed) + idx * np.uint64(0x9E3779B97F4A7C15)
+            z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+            z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+            z = z ^ (z >> np.uint64(31))
+        return z.view(np.uint8)[b0 - 8 * w0:b1 - 8 * w0].copy()
+    if kind in _BASES and n > _BASE_CAP[kind]:
+        base = np.frombuffer(_BASES[kind](_BASE_CAP[kind], seed), dtype=np.uint8)
+        out = np.empty(b1 - b0, dtype=np.uint8)
+        for dst, off, ln in _clip_plan(_segment_plan(base.size, n, seed), b0, b1):
+            out[dst:dst + ln] = base[off:off + ln]
+        return out
+    return generate(kind, n, seed)[b0:b1].copy()
+
+
+_DEV_BASE_CACHE: dict = {}
+
+
+def generate_range_device(kind: str, n: int, seed: int, b0: int, b1: int, device):
+    """generate_range on a CUDA device: tiled corpora upload their base corpus
+    once and gather the overlapping segments with device copies (SURVEY
+    §8(d): the 64 GiB config is built on the device from a host-made base);
+    other kinds are made on the host and uploaded.  Returns a uint8 tensor."""
+    import torch
+    if kind in _BASES and n > _BASE_CAP[kind]:
+        key = (kind, seed, str(device))
+        if key not in _DEV_BASE_CACHE:
+            base = np.frombuffer(_BASES[kind](_BASE_CAP[kind], seed), dtype=np.uint8)
+            _DEV_BASE_CACHE.clear()
+            _DEV_BASE_CACHE[key] = torch.from_numpy(base.copy()).to(device)
+        dbase = _DEV_BASE_CACHE[key]
+        out = torch.empty(b1 - b0, dtype=torch.uint8, device=device)
+        for dst, off, ln in _clip_plan(_segment_plan(dbase.numel(), n, seed), b0, b1):
+            out[dst:dst + ln].copy_(dbase[off:off + ln])
+        return out
+    return torch.from_numpy(generate_range(kind, n, seed, b0, b1)).to(device)
 
 
 # BASELINE.json configs (SURVEY §8(d)); sizes in bytes.

@@ -119,6 +119,13 @@ def compress_rank(x_slice, n_total: int, rank: int, world: int, S: int,
     return payload, sizes, placements(totals, n_total, S)[rank]
 
 
+def _global_rank(group, r: int) -> int:
+    """torch.distributed point-to-point and gather roots take GLOBAL ranks;
+    placements are indexed by the rank within `group`."""
+    import torch.distributed as dist
+    return r if group is None else dist.get_global_rank(group, r)
+
+
 def assemble_on_root(payload: bytes, sizes_le: bytes, place: RankPlacement, n_total: int,
                      params: Tuple[int, int, int, int], group=None):
     """Gather every rank's (table slice, payload) on rank 0 and build the
@@ -127,7 +134,7 @@ def assemble_on_root(payload: bytes, sizes_le: bytes, place: RankPlacement, n_to
     import torch.distributed as dist
     world = dist.get_world_size(group)
     objs = [None] * world if dist.get_rank(group) == 0 else None
-    dist.gather_object((place.rank, sizes_le, payload), objs, dst=0, group=group)
+    dist.gather_object((place.rank, sizes_le, payload), objs, dst=_global_rank(group, 0), group=group)
     if dist.get_rank(group) != 0:
         return None
     S, W, F, MIN = params
@@ -165,9 +172,9 @@ def assemble_on_root_tensors(payload, sizes, totals: Sequence[int], n_total: int
     if rank != 0:
         reqs = []
         if me.c1 > me.c0:
-            reqs.append(dist.isend(tab, dst=0, group=group))
+            reqs.append(dist.isend(tab, dst=_global_rank(group, 0), group=group))
         if me.payload_bytes:
-            reqs.append(dist.isend(payload.contiguous(), dst=0, group=group))
+            reqs.append(dist.isend(payload.contiguous(), dst=_global_rank(group, 0), group=group))
         for r in reqs:
             r.wait()
         return None
@@ -182,9 +189,9 @@ def assemble_on_root_tensors(payload, sizes, totals: Sequence[int], n_total: int
             psl.copy_(payload)
             continue
         if p.c1 > p.c0:
-            reqs.append(dist.irecv(tsl, src=p.rank, group=group))
+            reqs.append(dist.irecv(tsl, src=_global_rank(group, p.rank), group=group))
         if p.payload_bytes:
-            reqs.append(dist.irecv(psl, src=p.rank, group=group))
+            reqs.append(dist.irecv(psl, src=_global_rank(group, p.rank), group=group))
     for r in reqs:
         r.wait()
     return out
