@@ -66,5 +66,20 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+def build_int_peak(force: bool = False) -> str:
+    """tools/micro/int_peak: the integer-pipe microbenchmark bench.py runs for
+    the roofline's measured peak."""
+    src = os.path.join(ROOT, "tools", "micro", "int_peak.cu")
+    exe = os.path.join(ROOT, "tools", "micro", "int_peak")
+    if not force and os.path.exists(exe) and os.path.getmtime(exe) >= os.path.getmtime(src):
+        return exe
+    r = subprocess.run([NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-o", exe, src],
+                       capture_output=True, text=True)
+    if r.returncode != 0:
+        sys.stderr.write(r.stdout + r.stderr)
+        raise RuntimeError("nvcc failed on int_peak.cu")
+    return exe
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose=True))
