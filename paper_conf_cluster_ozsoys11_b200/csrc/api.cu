@@ -78,7 +78,11 @@ culzss_status check_params(const culzss_params *p, Geometry *g) {
     if (p->min_match != 3 || p->chunk_size < 1 || p->window < 1 || p->window > 256 ||
         p->max_match < 3 || p->max_match > 258 || p->reserved != 0)
         return CULZSS_ERR_INVALID_ARG;
-    if ((p->version != 0 && p->version != 2) || p->chunk_size > (uint32_t)kChunkMax || p->window > 255)
+    // W = 256 (the paper's "offsets are upto 256", PAPER.md:1@23151 §III.D):
+    // version 0 only, and F <= 256 (the walk's 16-bit token memo holds
+    // 256 x 254 match codes + literal + not-evaluated)
+    if ((p->version != 0 && p->version != 2) || p->chunk_size > (uint32_t)kChunkMax ||
+        (p->window == 256 && (p->version != 0 || p->max_match > 256)))
         return CULZSS_ERR_UNSUPPORTED;
     g->V = p->version;
     if (const char *e = getenv("CULZSS_WALK_SWITCH")) g->sw = (uint32_t)atol(e);

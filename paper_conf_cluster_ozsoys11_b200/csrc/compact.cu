@@ -147,7 +147,7 @@ compact_kernel(const uint8_t *__restrict__ bucket, uint64_t stride,
     const uint32_t nw = (uint32_t)((a1 - a0) >> 2);
     for (uint32_t j = lane; j < nw; j += 32) {
         const uint32_t s = head + 4 * j;            // source byte offset of this word
-        const uint32_t lo = s4[s >> 2], hi = s4[(s >> 2) + 1];
+        const uint32_t lo = s4[s >> 2], hi = (s & 3) ? s4[(s >> 2) + 1] : 0u;  // hi only when it is used
         o4[j] = __funnelshift_r(lo, hi, (s & 3) * 8);
     }
 }

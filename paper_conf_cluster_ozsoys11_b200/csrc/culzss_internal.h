@@ -78,7 +78,10 @@ struct __align__(16) WarpSmem {
     } a;
 };
 static_assert(sizeof(WarpSmem) <= 24848, "smem layout");
-static_assert(kChunkMax / 32 * 4 <= kStagePad, "run-boundary mask (one bit per position) fits in the staging pad");
+// a warp's run-boundary mask words (walk machine 2): its 64 + the 8 before
+// (run_start reaches back W <= 255) + the 9 after (run_len reaches F <= 258)
+constexpr int kBndWarpLo = 8, kBndWarpWords = 64 + kBndWarpLo + 9;
+static_assert(kWarpsPerChunk * kBndWarpWords * 4 <= kStagePad, "both warps' run-boundary masks fit in the staging pad");
 static_assert(offsetof(WarpSmem, a.u.w.xfer) - offsetof(WarpSmem, a.link) >= kWalkLanes * kStageWords * 4,
               "staging (over link + pad) must not reach xfer / ld");
 static_assert((kChunkMax * 9 / 8 + 16) <= sizeof(WarpSmem::a.u.w.ld), "payload words fit in ld");

@@ -50,9 +50,25 @@ namespace {
 constexpr uint32_t kFull = 0xffffffffu;
 constexpr uint32_t kTabBias = 0x1000;   // table entry = position + bias; 0 = empty
 constexpr uint32_t kHashMul = 0x9E3779B1u << 8;
-// memoised token encoding in ld[]: 0 = not evaluated, 2 = literal,
-// (D << 8) | (L - 3) = match (>= 0x100; L - 3 fits 8 bits for F <= 258)
-constexpr uint16_t kLit = 2;
+// Memoised token encoding in ld[] (u16).  W <= 128: 0 = not evaluated,
+// 2 = literal, (D << 8) | (L - 3) = match (>= 0x100; L - 3 fits 8 bits for
+// F <= 258).  W > 128 (BW; W = 256 needs D = 256): 0 = not evaluated,
+// 1 = literal, ((D - 1) << 8 | (L - 3)) + 2 = match, which fits 16 bits for
+// F <= 258 at W <= 255 and for F <= 256 at W = 256.
+template <bool BW>
+struct Memo {
+    static constexpr uint16_t kLit = BW ? 1 : 2;
+    __device__ static __forceinline__ uint32_t match(int D, int L) {
+        return BW ? ((((uint32_t)D - 1) << 8) | (uint32_t)(L - 3)) + 2u : ((uint32_t)D << 8) | (uint32_t)(L - 3);
+    }
+    __device__ static __forceinline__ bool is_match(uint32_t t) { return BW ? t >= 2 : t >= 0x100; }
+    // the token's 17 bits: flag 1 | D - 1 | L - 3 (reading R11)
+    __device__ static __forceinline__ uint32_t code(uint32_t t) {
+        return BW ? ((t - 2) | 0x10000u) : t + (0x10000u - 0x100u);
+    }
+    __device__ static __forceinline__ int len(uint32_t t) { return is_match(t) ? (int)(code(t) & 0xFF) + 3 : 1; }
+    __device__ static __forceinline__ int dist(uint32_t t) { return (int)((code(t) >> 8) & 0xFF) + 1; }
+};
 
 // skewed byte index of chunk position x (4 pad bytes per 128 positions)
 __device__ __forceinline__ int sk(int x) { return (int)((unsigned)x + (((unsigned)x >> 7) << 2)); }
@@ -103,7 +119,6 @@ __device__ __forceinline__ uint32_t hash_off(uint32_t w) { return ((w * kHashMul
 // the bank spread is the same as the interleaved layout's)
 __device__ __forceinline__ uint32_t hash9(uint32_t w) { return (w * kHashMul) >> 23; }
 
-__device__ __forceinline__ int tok_len(uint32_t t) { return t >= 0x100 ? (int)(t & 0xFF) + 3 : 1; }
 
 // Run-boundary mask (the run-skip prune): bit x of bnd (u32
 // words, position-indexed) = chunk[x] != chunk[x+1]; every bit from the
@@ -193,12 +208,14 @@ __device__ __forceinline__ int chain_after(const uint8_t *__restrict__ link, int
 
 // (L, D) at one position p by the chain walk with the same two exact prunes
 // as the walk state machine below (a plain loop: fix-up re-walks only).
-// m: end of p's chunk, cstart: its start.  Returns the memo encoding.
+// m: end of p's chunk, cstart: its start.  Returns the memo encoding.  At
+// W = 256 the links hold distances <= 255 and d = 256 is one extra candidate.
+template <bool BW>
 __device__ uint32_t eval_pos(const uint32_t *__restrict__ u, const uint8_t *__restrict__ link, int p, int m,
                              int cstart, int W, int F) {
     const int cap = min(F, m - p);
     int d = link[sk(p)];
-    if (cap < 3 || !d) return kLit;
+    if (cap < 3) return Memo<BW>::kLit;
     const int wlim = min(W, p - cstart);
     int t = -1;  // run length at p (computed when first needed)
     int bestL = 2, bestD = 0, o = 0, nrej = 0;
@@ -243,19 +260,26 @@ __device__ uint32_t eval_pos(const uint32_t *__restrict__ u, const uint8_t *__re
         const int l2 = link[sk(q + o)];
         d = (l2 && d + l2 <= wlim) ? d + l2 : 0;
     }
-    return bestD ? ((uint32_t)bestD << 8) | (uint32_t)(bestL - 3) : kLit;
+    if (BW && W == 256 && wlim == 256 && bestL < cap) {  // the one distance the u8 links cannot hold
+        const int L = lcp8(u, p - 256, p, cap);
+        if (L > bestL) {
+            bestL = L;
+            bestD = 256;
+        }
+    }
+    return bestD ? Memo<BW>::match(bestD, bestL) : Memo<BW>::kLit;
 }
 
-// Run-boundary mask of a warp's half of the chunk plus the 5 words each side
-// that run_len / run_start reach from it (positions [2048h - 160, 2048h +
-// 2208)), built on demand by the whole warp when it switches to the pruned
-// walk.  Both warps of a pair may write the shared words in between, with
-// identical values.  The skewed words of one 32-position group lie in one
-// 128-position segment; the group's next word is the pad word (a copy of the
-// next segment's first word) at a segment end.
+// Run-boundary mask of a warp's half of the chunk plus the words before and
+// after it that run_start / run_len reach from it (W <= 255 back, F <= 258
+// ahead: kBndWarpLo / kBndWarpWords), built on demand by the whole warp when it switches to the pruned
+// walk, into the warp's own copy (kBndWarpWords words; bnd points at its
+// word 0, so bnd[w] is mask word w).  The skewed words of one 32-position
+// group lie in one 128-position segment; the group's next word is the pad
+// word (a copy of the next segment's first word) at a segment end.
 __device__ __forceinline__ void build_bnd_warp(const uint32_t *__restrict__ cw, uint32_t *__restrict__ bnd,
                                                int half, int lane, int m) {
-    const int w0 = max(64 * half - 5, 0), w1 = min(64 * half + 69, kChunkMax / 32);
+    const int w0 = max(64 * half - kBndWarpLo, 0), w1 = min(64 * half + kBndWarpWords - kBndWarpLo, kChunkMax / 32);
 #pragma unroll 1
     for (int w = w0 + lane; w < w1; w += 32) {
         const uint32_t *c = cw + (sk(32 * w) >> 2);
@@ -308,7 +332,7 @@ __device__ __forceinline__ void build_bnd_warp(const uint32_t *__restrict__ cw, 
 // ALLPOS (per-position parity dump, row a2): every candidate position of the
 // segment is evaluated and (L, D) written to dump instead.
 // Returns the exit (first position >= s1 the greedy path reaches).
-template <bool ALLPOS>
+template <bool ALLPOS, bool BW>
 __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const uint8_t *__restrict__ link,
                                          const uint32_t *__restrict__ cw, uint32_t *__restrict__ bnd, uint64_t cm,
                                          uint16_t *__restrict__ ld, uint8_t *__restrict__ dump, int m, int mbuf,
@@ -323,10 +347,16 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
     bool active = p < s1;
     uint32_t nm = 0;  // matches found on the path
     int d = 0, cap = 0;
-    if (active) {
+    // W = 256: the links hold distances <= 255; d = 256 is evaluated as one
+    // extra candidate when the chain ends (t256: done), first if p has no link
+    bool t256 = false;
+    auto begin_token = [&]() {
         d = lks[p];
         cap = min(F, m - p);
-    }
+        t256 = BW && W == 256 && d == 0;
+        d = t256 ? 256 : d;
+    };
+    if (active) begin_token();
     int k = 0, bestL = 2, bestD = 0;
     int qr = 0;  // reject-test mode (int: no byte-register repacking)
     auto finish_token = [&]() {
@@ -334,20 +364,19 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
             dump[2 * p] = (uint8_t)(bestD ? bestL : 0);
             dump[2 * p + 1] = (uint8_t)bestD;
         } else {
-            lds[p] = (uint16_t)(bestD ? (bestD << 8) | (bestL - 3) : kLit);
+            lds[p] = (uint16_t)(bestD ? Memo<BW>::match(bestD, bestL) : Memo<BW>::kLit);
         }
         nm |= bestD;
         p = next_cand(cm, p + (ALLPOS ? 1 : (bestD ? bestL : 1)), s0, s1);
         active = p < s1;
-        if (active) {
-            d = lks[p];
-            cap = min(F, m - p);
-        }
+        if (active) begin_token();
         bestL = 2;
         bestD = 0;
         k = 0;
         qr = 0;
     };
+    // W = 256: when p's chain is exhausted, try d = 256 once
+    auto last256 = [&](bool fin) { return BW && fin && W == 256 && !t256 && bestL < cap && p - cstart >= 256; };
     // ---- machine 1: plain chain walk, until the warp has walked sw
     // iterations or one of its lanes has spent tx on its current token ------
     int it = 0, ti = 0;  // warp iterations, iterations of the lane's current token
@@ -376,8 +405,13 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
             bool tok_done = false;
             if (cand_done) {
                 const int l2 = bestL == cap ? 0 : lq;
-                const int nd = d + l2;
+                int nd = d + l2;
                 tok_done = l2 == 0 || nd > W;
+                if (last256(tok_done)) {
+                    tok_done = false;
+                    nd = 256;
+                    t256 = true;
+                }
                 d = nd;
                 k = 0;
                 qr = bestL >= 8 ? 1 : 0;
@@ -449,6 +483,13 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
                             fin = nd == 0;
                         }
                     }
+                    if (last256(fin)) {
+                        fin = false;
+                        nd = 256;
+                        o = 0;
+                        rs = 0;
+                        t256 = true;
+                    }
                     d = nd;
                     tok_done = fin;
                     k = 0;
@@ -474,6 +515,7 @@ __device__ __forceinline__ int walk_spec(const uint32_t *__restrict__ u, const u
 // there is the same.  A later re-walk of the same lane (rare: its entry moved
 // twice) cannot tell which earlier walk a memoised start belongs to and walks
 // to the segment end, reusing memoised tokens.
+template <bool BW>
 __device__ int walk_fix(const uint32_t *__restrict__ u, const uint8_t *__restrict__ link, uint64_t cm,
                         uint16_t *__restrict__ ld, int m, int cstart, int W, int F, int s0, int s1, int entry,
                         int spec_exit, bool first) {
@@ -484,10 +526,10 @@ __device__ int walk_fix(const uint32_t *__restrict__ u, const uint8_t *__restric
         uint32_t t = ld[sk2(p)];
         if (t && first) return spec_exit;
         if (!t) {
-            t = eval_pos(u, link, p, m, cstart, W, F);
+            t = eval_pos<BW>(u, link, p, m, cstart, W, F);
             ld[sk2(p)] = (uint16_t)t;
         }
-        p += tok_len(t);
+        p += Memo<BW>::len(t);
     }
 }
 
@@ -537,7 +579,8 @@ __device__ void v2_search_all(const uint32_t *cw, uint16_t *ld, int m, int W, in
             }
         }
         best = __reduce_max_sync(kFull, best);
-        if (lane == 0) ld[sk2(p)] = best ? (uint16_t)(((256 - (best & 0xFF)) << 8) | ((best >> 8) - 3)) : kLit;
+        if (lane == 0) ld[sk2(p)] = best ? (uint16_t)Memo<true>::match((int)(256 - (best & 0xFF)), (int)(best >> 8))
+                                         : Memo<true>::kLit;
     }
 }
 
@@ -545,7 +588,7 @@ __device__ void v2_search_all(const uint32_t *cw, uint16_t *ld, int m, int W, in
 // segment [.., s1); returns the exit (first position >= s1 on the path)
 __device__ __forceinline__ int v2_jump(const uint16_t *ld, int p, int s1) {
 #pragma unroll 1
-    while (p < s1) p += tok_len(ld[sk2(p)]);
+    while (p < s1) p += Memo<true>::len(ld[sk2(p)]);  // version 2 runs in the W > 128 instantiation
     return p;
 }
 
@@ -685,7 +728,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                                 uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(key));
                                 const uint32_t dist = (uint32_t)(p + j + kTabBias) - *e;
                                 *e = (uint16_t)(p + j + kTabBias);
-                                const bool ok = dist <= (uint32_t)W && (!PACK || dist <= (uint32_t)((p + j) & smask));
+                                // links are u8: distances <= 255 (W = 256 adds d = 256 in the walk)
+                                const bool ok = dist <= (uint32_t)min(W, 255) && (!PACK || dist <= (uint32_t)((p + j) & smask));
                                 lw |= (ok ? dist : 0u) << (8 * j);
                             }
                         }
@@ -713,8 +757,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
         for (int p = t64; p < m; p += kWalkLanes) {
             const uint32_t t = sm.a.u.w.ld[sk2(p)];
-            LD[2 * p] = (uint8_t)(t == kLit ? 0 : (t & 0xFF) + 3);
-            LD[2 * p + 1] = (uint8_t)(t == kLit ? 0 : t >> 8);
+            LD[2 * p] = (uint8_t)(Memo<true>::is_match(t) ? Memo<true>::len(t) : 0);
+            LD[2 * p + 1] = (uint8_t)(Memo<true>::is_match(t) ? Memo<true>::dist(t) : 0);
         }
         return;
     }
@@ -726,7 +770,8 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     const int cst = PACK ? (s0 & ~smask) : 0;  // start of the segment's chunk
     uint16_t *ld = sm.a.u.w.ld;
     uint32_t *ucw = sm.a.u.w.ucw;
-    uint32_t *bnd = reinterpret_cast<uint32_t *>(sm.a.u.w.pad);  // free until the bit-pack staging
+    // the warp's run-boundary mask (free until the bit-pack staging), indexed by mask word
+    uint32_t *bnd = reinterpret_cast<uint32_t *>(sm.a.u.w.pad) + kBndWarpWords * half + kBndWarpLo - 64 * half;
     if (!V2) {
         // zero the memoised tokens (their bytes held the hash tables) and
         // unskew the chunk for the walks' compares
@@ -754,6 +799,14 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
             const uint32_t nz = (((lw & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | lw) & 0x80808080u;
             h[w >> 3] |= ((nz >> 7) * 0x10204080u >> 28) << (4 * (w & 7));  // bit j = byte j nonzero
         }
+        if (!SMALLW && W == 256) {
+            // W = 256: a position whose 3-gram recurs exactly 256 back is a
+            // candidate too (the u8 links stop at 255; the walk adds d = 256)
+            for (int i = max(s0, cst + 256); i < min(s1, ce - 2); i++) {
+                if (((load4(sm.cw, i) ^ load4(sm.cw, i - 256)) & 0xFFFFFFu) == 0)
+                    h[(i - s0) >> 5] |= 1u << ((i - s0) & 31);
+            }
+        }
         if (s1 - s0 < 64) {  // positions >= s1 (garbage links)
             const int r = s1 - s0;
             h[0] &= r >= 32 ? 0xFFFFFFFFu : (1u << r) - 1;
@@ -768,12 +821,12 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     if (MODE == kModeDumpMatch) {
         // every candidate position through the production walk machine (a2)
         uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
-        walk_spec<true>(ucw, link, sm.cw, bnd, cm, ld, LD, ce, m, cst, W, F, s0, s1, half, lane, (int)g.sw,
+        walk_spec<true, !SMALLW>(ucw, link, sm.cw, bnd, cm, ld, LD, ce, m, cst, W, F, s0, s1, half, lane, (int)g.sw,
                         (int)g.tx, anym);
         return;
     }
     const int spec_exit =
-        V2 ? v2_jump(ld, s0, s1) : walk_spec<false>(ucw, link, sm.cw, bnd, cm, ld, nullptr, ce, m, cst, W, F, s0, s1, half, lane,
+        V2 ? v2_jump(ld, s0, s1) : walk_spec<false, !SMALLW>(ucw, link, sm.cw, bnd, cm, ld, nullptr, ce, m, cst, W, F, s0, s1, half, lane,
                                      (int)g.sw, (int)g.tx, anym);
     int exitp = spec_exit;
     int cur = s0;
@@ -802,7 +855,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         par ^= 1;
         if (chg) {
             exitp = V2 ? v2_jump(ld, entry, s1)
-                       : walk_fix(ucw, link, cm, ld, ce, cst, W, F, s0, s1, entry, spec_exit, first);
+                       : walk_fix<!SMALLW>(ucw, link, cm, ld, ce, cst, W, F, s0, s1, entry, spec_exit, first);
             first = false;
             cur = entry;
         }
@@ -818,8 +871,9 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                 p++;
             } else {
                 const uint32_t t = ld[sk2(p)];
-                tok[p] = t == kLit ? 1u : (((t & 0xFF) + 3) << 16) | (t >> 8);
-                p += tok_len(t);
+                tok[p] = Memo<!SMALLW>::is_match(t) ? ((uint32_t)Memo<!SMALLW>::len(t) << 16) | (uint32_t)Memo<!SMALLW>::dist(t)
+                                                    : 1u;
+                p += Memo<!SMALLW>::len(t);
             }
         }
         return;
@@ -882,10 +936,10 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                     const int p = s0 + 4 * i + j;
                     const uint32_t t = (j < 2 ? t01 : t23) >> (16 * (j & 1)) & 0xFFFFu;
                     const bool on = p >= cov && (!chk || p < s1);
-                    const bool mt = on && t >= 0x100;
+                    const bool mt = on && Memo<!SMALLW>::is_match(t);
                     const int nb = mt ? 17 : (on ? 9 : 0);
-                    const uint32_t val = mt ? t + (0x10000u - 0x100u) : (on ? (bytes >> (8 * j)) & 0xFFu : 0u);  // 1|D-1|L-3
-                    cov = mt ? p + (int)(t & 0xFF) + 3 : cov;
+                    const uint32_t val = mt ? Memo<!SMALLW>::code(t) : (on ? (bytes >> (8 * j)) & 0xFFu : 0u);  // 1|D-1|L-3
+                    cov = mt ? p + Memo<!SMALLW>::len(t) : cov;
                     pv = (pv << nb) | val;
                     pn += nb;
                     if (j & 1) {

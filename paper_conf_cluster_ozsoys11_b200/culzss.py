@@ -325,7 +325,8 @@ def match_search(x, params: Optional[Params] = None, stream=None):
     _check(_lib().culzss_match_search(ctypes.c_void_p(x.data_ptr()), x.numel(), ctypes.c_void_p(LD.data_ptr()),
                                       _params(params), _stream(stream)), "culzss_match_search")
     LD = LD[: 2 * x.numel()].view(-1, 2)
-    return LD[:, 0], LD[:, 1]
+    L, D = LD[:, 0], LD[:, 1].to(torch.int16)
+    return L, torch.where((L >= 3) & (D == 0), torch.full_like(D, 256), D)  # D byte 0 beside a match: D = 256
 
 
 def parse_tokens(x, params: Optional[Params] = None, stream=None):

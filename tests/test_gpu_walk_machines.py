@@ -135,3 +135,68 @@ def test_packed_small_chunks_each_machine(env, machine):
             x = run_inputs()[name]
             got = culzss.compress(dev(torch, x), p).cpu().numpy().tobytes()
             assert got == O.compress(x, S=S), (machine, name, S)
+
+
+@pytest.mark.parametrize("F", [3, 20, 128, 256])
+def test_window_256_streams(env, machine, F):
+    """W = 256 (PAPER.md:1@23151 §III.D "offsets are upto 256"): the u8 links
+    hold distances <= 255 and the walk evaluates d = 256 as one extra
+    candidate; byte-exact streams against the oracle, both machines."""
+    torch, culzss = env
+    p = culzss.Params.make(W=256, F=F)
+    rng = np.random.default_rng(256)
+    cases = dict(run_inputs())
+    for per in (127, 128, 200, 255, 256, 257):  # matches exactly at the window edge
+        base = rng.integers(0, 256, per, dtype=np.uint8)
+        cases[f"period{per}"] = np.tile(base, 3 * 4096 // per + 2)[:3 * 4096 + 11]
+    cases["csource"] = datagen.generate("csource", 3 * 4096 + 5, seed=31)
+    cases["random"] = datagen.generate("random", 2 * 4096, seed=32)
+    for name, x in cases.items():
+        got = culzss.compress(dev(torch, x), p).cpu().numpy().tobytes()
+        assert got == O.compress(x, W=256, F=F), (machine, name, F)
+
+
+def test_window_256_match_search(env, machine):
+    """Row a2 at W = 256: (L, D) at every position, including D = 256."""
+    torch, culzss = env
+    p = culzss.Params.make(W=256, F=200)
+    rng = np.random.default_rng(257)
+    xs = [np.tile(rng.integers(0, 256, 256, dtype=np.uint8), 20)[:2 * 4096 + 50],
+          datagen.generate("tarmix", 2 * 4096 + 9, seed=33), run_inputs()["runs20_alpha3"][:8192]]
+    seen256 = False
+    for x in xs:
+        L, D = culzss.match_search(dev(torch, x), p)
+        L, D = L.cpu().numpy(), D.cpu().numpy()
+        for c in range((x.size + 4095) // 4096):
+            chunk = x[c * 4096:(c + 1) * 4096]
+            eL, eD = O.match_all(chunk, W=256, F=200)
+            np.testing.assert_array_equal(L[c * 4096:c * 4096 + chunk.size], eL, err_msg=machine)
+            np.testing.assert_array_equal(D[c * 4096:c * 4096 + chunk.size], eD, err_msg=machine)
+            seen256 |= bool((eD == 256).any())
+    assert seen256  # the period-256 input exercises d = 256
+
+
+def test_window_256_packed_and_roundtrip(env, machine):
+    torch, culzss = env
+    for S in (512, 1024, 2048, 1000):
+        p = culzss.Params.make(S=S, W=256, F=256)
+        for name in ("runs20", "tarmix", "counters_step2"):
+            x = run_inputs()[name]
+            s = culzss.compress(dev(torch, x), p)
+            assert s.cpu().numpy().tobytes() == O.compress(x, S=S, W=256, F=256), (machine, name, S)
+            assert culzss.decompress(s).cpu().numpy().tobytes() == x.tobytes()
+
+
+def test_window_256_limits(env):
+    """W = 256 with F > 256 (the 16-bit token memo's code space) and version 2
+    at W = 256 are UNSUPPORTED; both stay valid parameters (INVALID_ARG is
+    for W > 256 / F > 258)."""
+    torch, culzss = env
+    x = dev(torch, datagen.generate("english", 5000, seed=1))
+    for kw in (dict(W=256, F=257), dict(W=256, F=258), dict(W=256, version=2)):
+        with pytest.raises(culzss.CulzssError) as e:
+            culzss.compress(x, culzss.Params.make(**kw))
+        assert e.value.status == culzss.ERR_UNSUPPORTED, kw
+    with pytest.raises(culzss.CulzssError) as e:
+        culzss.compress(x, culzss.Params.make(W=257))
+    assert e.value.status == culzss.ERR_INVALID_ARG
