@@ -81,7 +81,11 @@ culzss_status check_params(const culzss_params *p, Geometry *g) {
     // W = 256 (the paper's "offsets are upto 256", PAPER.md:1@23151 §III.D):
     // version 0 only, and F <= 256 (the walk's 16-bit token memo holds
     // 256 x 254 match codes + literal + not-evaluated)
-    if ((p->version != 0 && p->version != 2) || p->chunk_size > (uint32_t)kChunkMax ||
+    // S up to 64 KiB ("the decision on the length of the blocks is a
+    // configuration parameter", PAPER.md:1@30360 §V): version 0 compresses
+    // chunks above 4 KiB in tiles; version 2 is built for S <= 4096
+    if ((p->version != 0 && p->version != 2) || p->chunk_size > (uint32_t)kChunkTiledMax ||
+        (p->version == 2 && p->chunk_size > (uint32_t)kChunkMax) ||
         (p->window == 256 && (p->version != 0 || p->max_match > 256)))
         return CULZSS_ERR_UNSUPPORTED;
     g->V = p->version;

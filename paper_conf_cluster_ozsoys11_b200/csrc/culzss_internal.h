@@ -10,7 +10,8 @@
 namespace culzss {
 
 // Geometry of the fused chunk kernel.
-constexpr int kChunkMax = 4096;     // largest chunk the kernel stages (S <= 4096)
+constexpr int kChunkMax = 4096;     // the kernel's buffer: chunks of S <= 4096 in one piece
+constexpr int kChunkTiledMax = 1 << 16;  // S in (4096, 65536]: compressed in 4096-position tiles
 constexpr int kSeg = 128;           // positions per lane segment (32 x 128 = 4096)
 constexpr int kHashBits = 8;        // per-lane 3-gram hash table, W > 128: 256 u16 heads
 constexpr int kHashBitsSmallW = 9;  // W <= 128: 512 u8 heads (relative positions)

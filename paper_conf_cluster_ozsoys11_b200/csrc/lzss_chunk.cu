@@ -596,7 +596,7 @@ __device__ __forceinline__ void pair_sync(int id) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(kWalkLanes) : "memory");
 }
 
-template <int MODE, bool SMALLW, bool V2, bool PACK>
+template <int MODE, bool SMALLW, bool V2, bool PACK, bool TILED>
 __global__ void __launch_bounds__(kChunksPerCta * kWalkLanes, kCtasPerSm)
 chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__restrict__ bucket,
              uint32_t *__restrict__ sizes, void *__restrict__ dbg) {
@@ -616,449 +616,496 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
     asm volatile("griddepcontrol.launch_dependents;");
     if (c >= C) return;  // both warps of the pair leave together
     const uint64_t start = c * g.S;
-    const int m = (int)min((uint64_t)g.K * g.S, n - start);
+    // !TILED: the buffer's length (one chunk, or K packed small chunks);
+    // TILED: the chunk's length (S > 4096)
+    const int m0 = (int)min((uint64_t)g.K * g.S, n - start);
     const int smask = PACK ? (int)g.smask : 4095;  // !PACK: one chunk, no inner bounds
     const int W = g.W, F = g.F;
-    const uint8_t *src = in + start;
     uint8_t *cb = reinterpret_cast<uint8_t *>(sm.cw);
     uint8_t *link = sm.a.link;
-
-    // ---------------- a1: stage the chunk (16-byte coalesced loads) --------
-    // a full chunk overwrites every data byte, so nothing needs clearing and
-    // no barrier has to order the clearing before the data stores (bytes past
-    // the chunk end are only ever read beyond a match's cap)
-    const bool full = m == kChunkMax;
-    {
-        uint4 *z4 = reinterpret_cast<uint4 *>(sm.cw);
-        const uint4 z = make_uint4(0, 0, 0, 0);
-        if (!full) {
-            for (int i = t64; i < (int)(sizeof(sm.cw) / 16); i += kWalkLanes) z4[i] = z;
-        }
-        uint4 *t4 = reinterpret_cast<uint4 *>(sm.a.u.tab);
-        // u8 tables: empty = (s0 - 129) mod 256 = 0x7F (even lanes) / 0xFF (odd)
-#pragma unroll 4
-        for (int i = t64; i < (int)(sizeof(sm.a.u.tab) / 16); i += kWalkLanes) {
-            // u8 tables: lane (i >> 5)'s 512 bytes hold its empty value
-            const uint32_t e = SMALLW ? ((i >> 5) & 1 ? 0xFFFFFFFFu : 0x7F7F7F7Fu) : 0u;
-            t4[i] = make_uint4(e, e, e, e);
-        }
-    }
-    if (!full) pair_sync(bar);  // (uniform per pair)
-    if ((reinterpret_cast<uintptr_t>(src) & 15) == 0) {
-        // a 16-byte group never straddles a 128-position segment
-        const int nvec = m >> 4;
-        const uint4 *s4 = reinterpret_cast<const uint4 *>(src);
-#pragma unroll 4
-        for (int i = t64; i < nvec; i += kWalkLanes) {
-            const uint4 v = __ldcs(s4 + i);
-            uint32_t *d = sm.cw + (sk(i << 4) >> 2);
-            d[0] = v.x;
-            d[1] = v.y;
-            d[2] = v.z;
-            d[3] = v.w;
-        }
-        for (int i = (nvec << 4) + t64; i < m; i += kWalkLanes) cb[sk(i)] = src[i];
-    } else {
-        for (int i = t64; i < m; i += kWalkLanes) cb[sk(i)] = src[i];
-    }
-    pair_sync(bar);
-    // pad word of 128-segment `lane` = first word of the next segment (0 past the end)
-    if (half == 0) sm.cw[33 * lane + 32] = lane < 31 ? sm.cw[33 * (lane + 1)] : 0u;
-    pair_sync(bar);
-
-    // ---------------- a2 part 1: per-lane 3-gram hash chains (warp 0) ------
-    // Lane l of warp 0 owns the 128-position build segment [128 l, 128 l + 128)
-    // and its own hash table; straight-line: every position is hashed and
-    // inserted; the last two positions (no 3-gram) get link 0 after.
-    if (!V2 && half == 0) {
-        const int b0 = lane * kSeg;
-        const int b1 = min(b0 + kSeg, m);
-        unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + (SMALLW ? 512 * lane : 2 * lane);
-        if (b0 < m) {
-            // the W positions before the segment (pre-insert, no links)
-#pragma unroll 4
-            for (int q = max(0, b0 - W) & ~3; q < b0; q += 4) {
-                const uint32_t w0 = sm.cw[sk(q) >> 2], w1 = sm.cw[(sk(q) >> 2) + 1];
-#pragma unroll
-                for (int j = 0; j < 4; j++) {
-                    const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
-                    if (SMALLW)
-                        tabl[hash9(key)] = (uint8_t)(q + j);
-                    else
-                        *reinterpret_cast<uint16_t *>(tabl + hash_off(key)) = (uint16_t)(q + j + kTabBias);
-                }
-            }
-            // own segment: links
-            const uint32_t w4 = (uint32_t)min(W, 255) * 0x01010101u;
+    // TILED (S > 4096; DESIGN.md §5 "large chunks"): the chunk is compressed
+    // in tiles of one 4096-position buffer each -- chunk bytes [B0, B0 + m),
+    // B0 = the tile's first parse position minus Hh >= W bytes of window
+    // history; parse region [T0, T1) in buffer coordinates (the last Fh >= F - 1
+    // positions of a non-last tile are lookahead only); the greedy path enters
+    // the tile at Eb and leaves it at the first position >= T1 it reaches.  The
+    // tiles' bits are appended to the chunk's bucket 16-byte unit by unit; the
+    // last partial unit is carried to the next tile.
+    const int Hh = TILED ? (W + 63) & ~63 : 0, Fh = TILED ? (F - 1 + 63) & ~63 : 0;
+    int tileT1c = 0, Ec = 0;  // previous tile's parse end, the path's entry (chunk coordinates)
+    int boff = 0;             // payload bits of the earlier tiles
+    uint32_t cy0 = 0, cy1 = 0, cy2 = 0, cy3 = 0;  // their last, partial 16-byte unit (payload words)
 #pragma unroll 1
-            for (int wi = 0; wi < 4; wi++) {
-                const int pb = b0 + 32 * wi;
-                if (pb < b1) {
-#pragma unroll
-                    for (int i = 0; i < 8; i++) {
-                        const int p = pb + 4 * i;
-                        const uint32_t w0 = sm.cw[sk(p) >> 2], w1 = sm.cw[(sk(p) >> 2) + 1];
-                        uint32_t lw = 0;
-                        if (SMALLW) {
-                            // entries hold position mod 256: every live entry is
-                            // within 256 of p, the empty value maps to 0 or > 128.
-                            // Entries are read and replaced in position order
-                            // (a repeated hash in the group sees its predecessor),
-                            // then the four distances are formed bytewise.
-                            uint32_t E = 0;
-#pragma unroll
-                            for (int j = 0; j < 4; j++) {
-                                uint8_t *e = tabl + hash9(__funnelshift_r(w0, w1, 8 * j));
-                                E |= (uint32_t)*e << (8 * j);
-                                *e = (uint8_t)(p + j);
-                            }
-                            const uint32_t D = __vsub4(__vadd4(((uint32_t)p & 0xFFu) * 0x01010101u, 0x03020100u), E);
-                            // at most W, and never before the chunk start (packed
-                            // small chunks; a 4-group lies in one chunk)
-                            uint32_t lim = w4;
-                            if (PACK) {
-                                const uint32_t rel = (uint32_t)min(p & smask, 252);
-                                lim = __vminu4(w4, __vadd4(rel * 0x01010101u, 0x03020100u));
-                            }
-                            lw = D & __vcmpleu4(D, lim);  // distance, or 0 past the window
-                        } else {
-#pragma unroll
-                            for (int j = 0; j < 4; j++) {
-                                const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
-                                uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(key));
-                                const uint32_t dist = (uint32_t)(p + j + kTabBias) - *e;
-                                *e = (uint16_t)(p + j + kTabBias);
-                                // links are u8: distances <= 255 (W = 256 adds d = 256 in the walk)
-                                const bool ok = dist <= (uint32_t)min(W, 255) && (!PACK || dist <= (uint32_t)((p + j) & smask));
-                                lw |= (ok ? dist : 0u) << (8 * j);
-                            }
-                        }
-                        *reinterpret_cast<uint32_t *>(link + sk(p)) = lw;
-                    }
-                }
-            }
-        }
-        // positions m-2 and m-1 have no 3-gram: never candidates
-#pragma unroll
-        for (int t = 1; t <= 2; t++) {
-            const int x = m - t;
-            if (x >= b0 && x < b1) link[sk(x)] = 0;
-        }
-    }
-    pair_sync(bar);  // tab is dead from here on
-    if (V2) {
-        // version 2: (L, D) of every position by the warp-cooperative search
-        v2_search_all(sm.cw, sm.a.u.w.ld, m, W, F, half, lane, smask);
-        pair_sync(bar);
-    }
+    for (int tile = 0;; tile++) {
+        if (TILED && tile > 0) pair_sync(bar);  // the previous tile's shared-memory reads are done
+        const int B0 = TILED && tile > 0 ? tileT1c - Hh : 0;
+        const int m = TILED ? min(kChunkMax, m0 - B0) : m0;
+        const bool last = !TILED || m0 - B0 <= kChunkMax;
+        const int T0 = TILED && tile > 0 ? Hh : 0;
+        const int T1 = last ? m : kChunkMax - Fh;
+        const int Eb = Ec - B0;
+        const uint8_t *src = in + start + B0;
 
-    if (V2 && MODE == kModeDumpMatch) {
-        // every position's evaluated token, for per-position parity (a2)
-        uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
-        for (int p = t64; p < m; p += kWalkLanes) {
-            const uint32_t t = sm.a.u.w.ld[sk2(p)];
-            LD[2 * p] = (uint8_t)(Memo<true>::is_match(t) ? Memo<true>::len(t) : 0);
-            LD[2 * p + 1] = (uint8_t)(Memo<true>::is_match(t) ? Memo<true>::dist(t) : 0);
-        }
-        return;
-    }
-
-    // ---------------- a3: lazy greedy walk, speculative per 64-segment -----
-    const int s0 = t64 * kWSeg;
-    const int s1 = min(s0 + kWSeg, m);  // <= s0 for lanes past the chunk end
-    const int ce = PACK ? min((s0 | smask) + 1, m) : m;  // end of the segment's chunk (matches stop there)
-    const int cst = PACK ? (s0 & ~smask) : 0;  // start of the segment's chunk
-    uint16_t *ld = sm.a.u.w.ld;
-    uint32_t *ucw = sm.a.u.w.ucw;
-    // the warp's run-boundary mask (free until the bit-pack staging), indexed by mask word
-    uint32_t *bnd = reinterpret_cast<uint32_t *>(sm.a.u.w.pad) + kBndWarpWords * half + kBndWarpLo - 64 * half;
-    if (!V2) {
-        // zero the memoised tokens (their bytes held the hash tables) and
-        // unskew the chunk for the walks' compares
-        uint4 *l4 = reinterpret_cast<uint4 *>(ld);
-        const uint4 z = make_uint4(0, 0, 0, 0);
-#pragma unroll 4
-        for (int i = t64; i < (int)(sizeof(sm.a.u.w.ld) / 16); i += kWalkLanes) l4[i] = z;
-#pragma unroll 4
-        for (int j = t64; j < kUcwWords; j += kWalkLanes)
-            ucw[j] = j < kChunkMax / 4 ? __byte_perm(sm.cw[j + (j >> 5)], 0, 0x0123) : 0u;  // + zero tail
-    }
-    // candidate mask: bit i = position s0 + i (< s1) has a chain link
-    uint32_t rc0 = 0, rc1 = 0;
-    if (V2) {
-        // every position holds its evaluated token
-        const int r = max(s1 - s0, 0);
-        rc0 = r >= 32 ? 0xFFFFFFFFu : ~(0xFFFFFFFFu >> r);
-        rc1 = r <= 32 ? 0u : (r >= 64 ? 0xFFFFFFFFu : ~(0xFFFFFFFFu >> (r - 32)));
-    } else if (s0 < s1) {
-        const int so = (s0 >> 7) << 2;  // constant skew inside the segment
-        uint32_t h[2] = {0, 0};
-#pragma unroll
-        for (int w = 0; w < kWSeg / 4; w++) {
-            const uint32_t lw = *reinterpret_cast<const uint32_t *>(link + so + s0 + 4 * w);
-            const uint32_t nz = (((lw & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | lw) & 0x80808080u;
-            h[w >> 3] |= ((nz >> 7) * 0x10204080u >> 28) << (4 * (w & 7));  // bit j = byte j nonzero
-        }
-        if (!SMALLW && W == 256) {
-            // W = 256: a position whose 3-gram recurs exactly 256 back is a
-            // candidate too (the u8 links stop at 255; the walk adds d = 256)
-            for (int i = max(s0, cst + 256); i < min(s1, ce - 2); i++) {
-                if (((load4(sm.cw, i) ^ load4(sm.cw, i - 256)) & 0xFFFFFFu) == 0)
-                    h[(i - s0) >> 5] |= 1u << ((i - s0) & 31);
+        // ---------------- a1: stage the chunk (16-byte coalesced loads) --------
+        // a full chunk overwrites every data byte, so nothing needs clearing and
+        // no barrier has to order the clearing before the data stores (bytes past
+        // the chunk end are only ever read beyond a match's cap)
+        const bool full = m == kChunkMax;
+        {
+            uint4 *z4 = reinterpret_cast<uint4 *>(sm.cw);
+            const uint4 z = make_uint4(0, 0, 0, 0);
+            if (!full) {
+                for (int i = t64; i < (int)(sizeof(sm.cw) / 16); i += kWalkLanes) z4[i] = z;
+            }
+            uint4 *t4 = reinterpret_cast<uint4 *>(sm.a.u.tab);
+            // u8 tables: empty = (s0 - 129) mod 256 = 0x7F (even lanes) / 0xFF (odd)
+    #pragma unroll 4
+            for (int i = t64; i < (int)(sizeof(sm.a.u.tab) / 16); i += kWalkLanes) {
+                // u8 tables: lane (i >> 5)'s 512 bytes hold its empty value
+                const uint32_t e = SMALLW ? ((i >> 5) & 1 ? 0xFFFFFFFFu : 0x7F7F7F7Fu) : 0u;
+                t4[i] = make_uint4(e, e, e, e);
             }
         }
-        if (s1 - s0 < 64) {  // positions >= s1 (garbage links)
-            const int r = s1 - s0;
-            h[0] &= r >= 32 ? 0xFFFFFFFFu : (1u << r) - 1;
-            h[1] &= r <= 32 ? 0u : (1u << (r - 32)) - 1;
-        }
-        rc0 = __brev(h[0]);
-        rc1 = __brev(h[1]);
-    }
-    pair_sync(bar);
-    bool anym = true;  // the speculative path holds a match (V2: not tracked)
-    const uint64_t cm = ((uint64_t)rc0 << 32) | rc1;
-    if (MODE == kModeDumpMatch) {
-        // every candidate position through the production walk machine (a2)
-        uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
-        walk_spec<true, !SMALLW>(ucw, link, sm.cw, bnd, cm, ld, LD, ce, m, cst, W, F, s0, s1, half, lane, (int)g.sw,
-                        (int)g.tx, anym);
-        return;
-    }
-    const int spec_exit =
-        V2 ? v2_jump(ld, s0, s1) : walk_spec<false, !SMALLW>(ucw, link, sm.cw, bnd, cm, ld, nullptr, ce, m, cst, W, F, s0, s1, half, lane,
-                                     (int)g.sw, (int)g.tx, anym);
-    int exitp = spec_exit;
-    int cur = s0;
-    bool first = true;
-    volatile uint32_t *xf = sm.a.u.w.xfer;
-    // two barriers per round: exits and "changed" flags use slots alternating
-    // with the round's parity, so a slot is rewritten only two rounds later,
-    // after every read of it
-    int par = 0;
-#pragma unroll 1
-    while (true) {
-        // entry of walk lane t64 = exit of lane t64 - 1 (warp 1 lane 0 reads
-        // warp 0 lane 31 through shared memory)
-        int entry = __shfl_up_sync(kFull, exitp, 1);
-        if (lane == 31) xf[2 * par + half] = (uint32_t)exitp;
-        pair_sync(bar);
-        if (lane == 0) entry = half ? (int)xf[2 * par + half - 1] : 0;
-        const bool chg = entry != cur;
-        const bool any = __any_sync(kFull, chg);
-        if (lane == 0) xf[4 + 2 * par + half] = any;
-        pair_sync(bar);
-        bool go = false;
-#pragma unroll
-        for (int k = 0; k < kWarpsPerChunk; k++) go |= xf[4 + 2 * par + k] != 0;
-        if (!go) break;
-        par ^= 1;
-        if (chg) {
-            exitp = V2 ? v2_jump(ld, entry, s1)
-                       : walk_fix<!SMALLW>(ucw, link, cm, ld, ce, cst, W, F, s0, s1, entry, spec_exit, first);
-            first = false;
-            cur = entry;
-        }
-    }
-
-    if (MODE == kModeDumpTokens) {
-        uint32_t *tok = reinterpret_cast<uint32_t *>(dbg) + start;
-        for (int p = s0; p < s1; p++) tok[p] = 0;
-        int p = cur;
-        while (p < s1) {
-            if (!is_cand(cm, p - s0)) {
-                tok[p] = 1;
-                p++;
-            } else {
-                const uint32_t t = ld[sk2(p)];
-                tok[p] = Memo<!SMALLW>::is_match(t) ? ((uint32_t)Memo<!SMALLW>::len(t) << 16) | (uint32_t)Memo<!SMALLW>::dist(t)
-                                                    : 1u;
-                p += Memo<!SMALLW>::len(t);
+        if (!full) pair_sync(bar);  // (uniform per pair)
+        if ((reinterpret_cast<uintptr_t>(src) & 15) == 0) {
+            // a 16-byte group never straddles a 128-position segment
+            const int nvec = m >> 4;
+            const uint4 *s4 = reinterpret_cast<const uint4 *>(src);
+    #pragma unroll 4
+            for (int i = t64; i < nvec; i += kWalkLanes) {
+                const uint4 v = __ldcs(s4 + i);
+                uint32_t *d = sm.cw + (sk(i << 4) >> 2);
+                d[0] = v.x;
+                d[1] = v.y;
+                d[2] = v.z;
+                d[3] = v.w;
             }
-        }
-        return;
-    }
-    pair_sync(bar);  // link is dead: staging may overwrite it
-
-    // ---------------- a4: bit-pack ----------------------------------------
-    // Each walk lane emits its path's tokens MSB-first into its own staging
-    // words starting at bit 0 (a token is up to 3 literals of a candidate-free
-    // run, an evaluated literal, or a match); after the scan of bit counts the
-    // staged words are shifted into place.
-    uint32_t *stage = reinterpret_cast<uint32_t *>(sm.a.link) + t64 * kStageWords;
-    int nbits = 0;
-    {
-        // Uniform position scan (no token jumps): every position >= the lane's
-        // true entry is either inside a path match (covered) or a path token
-        // start; a token start's memoised ld[] is its token whichever walk
-        // wrote it, and is 0 for candidate-free positions (literals).  Each
-        // position emits 0, 9 or 17 bits.
-        uint64_t acc = 0;
-        int nacc = 0;
-        uint32_t *sp = stage;  // next staging word
-        int cov = cur;  // positions < cov are covered (by the previous lane or a match)
-        const int so = (s0 >> 7) << 2;
-        const uint32_t *ldw = reinterpret_cast<const uint32_t *>(ld + (so >> 1) + s0);  // 2 tokens / word
-        const uint32_t *cbw = reinterpret_cast<const uint32_t *>(cb + so + s0);         // 4 bytes / word
-        const int ng = (s1 - s0 + 3) >> 2;
-        // append pn (<= 26) bits; acc keeps < 32 pending bits between calls
-        auto put = [&](uint32_t pv, int pn) {
-            acc = (acc << pn) | pv;
-            nacc += pn;
-            if (nacc >= 32) {
-                nacc -= 32;
-                *sp++ = (uint32_t)(acc >> nacc);
-            }
-        };
-        if (__all_sync(kFull, !anym && cur == s0 && s1 - s0 == kWSeg)) {
-            // every lane of the warp walks its whole segment from its start
-            // and found no match: 64 literals each (incompressible data),
-            // emitted branch-free in 18-bit pairs (bit positions static)
-#pragma unroll
-            for (int i = 0; i < kWSeg / 4; i++) {
-                const uint32_t bytes = cbw[i];
-                put(((bytes & 0xFFu) << 9) | ((bytes >> 8) & 0xFFu), 18);
-                put((((bytes >> 16) & 0xFFu) << 9) | (bytes >> 24), 18);
-            }
+            for (int i = (nvec << 4) + t64; i < m; i += kWalkLanes) cb[sk(i)] = src[i];
         } else {
-            // groups wholly inside a match are skipped.  Positions are
-            // combined in pairs in 32 bits first: a pair is at most a literal
-            // and a match (26 bits), since a match covers the next position.
-            // Only a chunk's last lane can have a partial last group: full
-            // groups skip the segment-end test.
-            auto group = [&](int i, bool chk) {
-                const uint32_t bytes = cbw[i];
-                const uint32_t t01 = ldw[2 * i], t23 = ldw[2 * i + 1];
-                uint32_t pv = 0;
-                int pn = 0;
-#pragma unroll
-                for (int j = 0; j < 4; j++) {
-                    const int p = s0 + 4 * i + j;
-                    const uint32_t t = (j < 2 ? t01 : t23) >> (16 * (j & 1)) & 0xFFFFu;
-                    const bool on = p >= cov && (!chk || p < s1);
-                    const bool mt = on && Memo<!SMALLW>::is_match(t);
-                    const int nb = mt ? 17 : (on ? 9 : 0);
-                    const uint32_t val = mt ? Memo<!SMALLW>::code(t) : (on ? (bytes >> (8 * j)) & 0xFFu : 0u);  // 1|D-1|L-3
-                    cov = mt ? p + Memo<!SMALLW>::len(t) : cov;
-                    pv = (pv << nb) | val;
-                    pn += nb;
-                    if (j & 1) {
-                        put(pv, pn);
-                        pv = 0;
-                        pn = 0;
+            for (int i = t64; i < m; i += kWalkLanes) cb[sk(i)] = src[i];
+        }
+        pair_sync(bar);
+        // pad word of 128-segment `lane` = first word of the next segment (0 past the end)
+        if (half == 0) sm.cw[33 * lane + 32] = lane < 31 ? sm.cw[33 * (lane + 1)] : 0u;
+        pair_sync(bar);
+
+        // ---------------- a2 part 1: per-lane 3-gram hash chains (warp 0) ------
+        // Lane l of warp 0 owns the 128-position build segment [128 l, 128 l + 128)
+        // and its own hash table; straight-line: every position is hashed and
+        // inserted; the last two positions (no 3-gram) get link 0 after.
+        if (!V2 && half == 0) {
+            const int b0 = lane * kSeg;
+            const int b1 = min(b0 + kSeg, m);
+            unsigned char *tabl = reinterpret_cast<unsigned char *>(sm.a.u.tab) + (SMALLW ? 512 * lane : 2 * lane);
+            if (b0 < m) {
+                // the W positions before the segment (pre-insert, no links)
+    #pragma unroll 4
+                for (int q = max(0, b0 - W) & ~3; q < b0; q += 4) {
+                    const uint32_t w0 = sm.cw[sk(q) >> 2], w1 = sm.cw[(sk(q) >> 2) + 1];
+    #pragma unroll
+                    for (int j = 0; j < 4; j++) {
+                        const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
+                        if (SMALLW)
+                            tabl[hash9(key)] = (uint8_t)(q + j);
+                        else
+                            *reinterpret_cast<uint16_t *>(tabl + hash_off(key)) = (uint16_t)(q + j + kTabBias);
                     }
+                }
+                // own segment: links
+                const uint32_t w4 = (uint32_t)min(W, 255) * 0x01010101u;
+    #pragma unroll 1
+                for (int wi = 0; wi < 4; wi++) {
+                    const int pb = b0 + 32 * wi;
+                    if (pb < b1) {
+    #pragma unroll
+                        for (int i = 0; i < 8; i++) {
+                            const int p = pb + 4 * i;
+                            const uint32_t w0 = sm.cw[sk(p) >> 2], w1 = sm.cw[(sk(p) >> 2) + 1];
+                            uint32_t lw = 0;
+                            if (SMALLW) {
+                                // entries hold position mod 256: every live entry is
+                                // within 256 of p, the empty value maps to 0 or > 128.
+                                // Entries are read and replaced in position order
+                                // (a repeated hash in the group sees its predecessor),
+                                // then the four distances are formed bytewise.
+                                uint32_t E = 0;
+    #pragma unroll
+                                for (int j = 0; j < 4; j++) {
+                                    uint8_t *e = tabl + hash9(__funnelshift_r(w0, w1, 8 * j));
+                                    E |= (uint32_t)*e << (8 * j);
+                                    *e = (uint8_t)(p + j);
+                                }
+                                const uint32_t D = __vsub4(__vadd4(((uint32_t)p & 0xFFu) * 0x01010101u, 0x03020100u), E);
+                                // at most W, and never before the chunk start (packed
+                                // small chunks; a 4-group lies in one chunk)
+                                uint32_t lim = w4;
+                                if (PACK) {
+                                    const uint32_t rel = (uint32_t)min(p & smask, 252);
+                                    lim = __vminu4(w4, __vadd4(rel * 0x01010101u, 0x03020100u));
+                                }
+                                lw = D & __vcmpleu4(D, lim);  // distance, or 0 past the window
+                            } else {
+    #pragma unroll
+                                for (int j = 0; j < 4; j++) {
+                                    const uint32_t key = __funnelshift_r(w0, w1, 8 * j);
+                                    uint16_t *e = reinterpret_cast<uint16_t *>(tabl + hash_off(key));
+                                    const uint32_t dist = (uint32_t)(p + j + kTabBias) - *e;
+                                    *e = (uint16_t)(p + j + kTabBias);
+                                    // links are u8: distances <= 255 (W = 256 adds d = 256 in the walk)
+                                    const bool ok = dist <= (uint32_t)min(W, 255) && (!PACK || dist <= (uint32_t)((p + j) & smask));
+                                    lw |= (ok ? dist : 0u) << (8 * j);
+                                }
+                            }
+                            *reinterpret_cast<uint32_t *>(link + sk(p)) = lw;
+                        }
+                    }
+                }
+            }
+            // positions m-2 and m-1 have no 3-gram: never candidates
+    #pragma unroll
+            for (int t = 1; t <= 2; t++) {
+                const int x = m - t;
+                if (x >= b0 && x < b1) link[sk(x)] = 0;
+            }
+        }
+        pair_sync(bar);  // tab is dead from here on
+        if (V2) {
+            // version 2: (L, D) of every position by the warp-cooperative search
+            v2_search_all(sm.cw, sm.a.u.w.ld, m, W, F, half, lane, smask);
+            pair_sync(bar);
+        }
+
+        if (V2 && MODE == kModeDumpMatch) {
+            // every position's evaluated token, for per-position parity (a2)
+            uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * start;
+            for (int p = t64; p < m; p += kWalkLanes) {
+                const uint32_t t = sm.a.u.w.ld[sk2(p)];
+                LD[2 * p] = (uint8_t)(Memo<true>::is_match(t) ? Memo<true>::len(t) : 0);
+                LD[2 * p + 1] = (uint8_t)(Memo<true>::is_match(t) ? Memo<true>::dist(t) : 0);
+            }
+            return;
+        }
+
+        // ---------------- a3: lazy greedy walk, speculative per 64-segment -----
+        const int s0 = t64 * kWSeg;
+        // <= s0 for lanes past the chunk end (TILED: outside the parse region)
+        const int s1 = TILED ? (s0 >= T0 && s0 < T1 ? min(s0 + kWSeg, T1) : s0) : min(s0 + kWSeg, m);
+        const int ce = PACK ? min((s0 | smask) + 1, m) : m;  // end of the segment's chunk (matches stop there)
+        const int cst = PACK ? (s0 & ~smask) : 0;  // start of the segment's chunk
+        uint16_t *ld = sm.a.u.w.ld;
+        uint32_t *ucw = sm.a.u.w.ucw;
+        // the warp's run-boundary mask (free until the bit-pack staging), indexed by mask word
+        uint32_t *bnd = reinterpret_cast<uint32_t *>(sm.a.u.w.pad) + kBndWarpWords * half + kBndWarpLo - 64 * half;
+        if (!V2) {
+            // zero the memoised tokens (their bytes held the hash tables) and
+            // unskew the chunk for the walks' compares
+            uint4 *l4 = reinterpret_cast<uint4 *>(ld);
+            const uint4 z = make_uint4(0, 0, 0, 0);
+    #pragma unroll 4
+            for (int i = t64; i < (int)(sizeof(sm.a.u.w.ld) / 16); i += kWalkLanes) l4[i] = z;
+    #pragma unroll 4
+            for (int j = t64; j < kUcwWords; j += kWalkLanes)
+                ucw[j] = j < kChunkMax / 4 ? __byte_perm(sm.cw[j + (j >> 5)], 0, 0x0123) : 0u;  // + zero tail
+        }
+        // candidate mask: bit i = position s0 + i (< s1) has a chain link
+        uint32_t rc0 = 0, rc1 = 0;
+        if (V2) {
+            // every position holds its evaluated token
+            const int r = max(s1 - s0, 0);
+            rc0 = r >= 32 ? 0xFFFFFFFFu : ~(0xFFFFFFFFu >> r);
+            rc1 = r <= 32 ? 0u : (r >= 64 ? 0xFFFFFFFFu : ~(0xFFFFFFFFu >> (r - 32)));
+        } else if (s0 < s1) {
+            const int so = (s0 >> 7) << 2;  // constant skew inside the segment
+            uint32_t h[2] = {0, 0};
+    #pragma unroll
+            for (int w = 0; w < kWSeg / 4; w++) {
+                const uint32_t lw = *reinterpret_cast<const uint32_t *>(link + so + s0 + 4 * w);
+                const uint32_t nz = (((lw & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | lw) & 0x80808080u;
+                h[w >> 3] |= ((nz >> 7) * 0x10204080u >> 28) << (4 * (w & 7));  // bit j = byte j nonzero
+            }
+            if (!SMALLW && W == 256) {
+                // W = 256: a position whose 3-gram recurs exactly 256 back is a
+                // candidate too (the u8 links stop at 255; the walk adds d = 256)
+                for (int i = max(s0, cst + 256); i < min(s1, ce - 2); i++) {
+                    if (((load4(sm.cw, i) ^ load4(sm.cw, i - 256)) & 0xFFFFFFu) == 0)
+                        h[(i - s0) >> 5] |= 1u << ((i - s0) & 31);
+                }
+            }
+            if (s1 - s0 < 64) {  // positions >= s1 (garbage links)
+                const int r = s1 - s0;
+                h[0] &= r >= 32 ? 0xFFFFFFFFu : (1u << r) - 1;
+                h[1] &= r <= 32 ? 0u : (1u << (r - 32)) - 1;
+            }
+            rc0 = __brev(h[0]);
+            rc1 = __brev(h[1]);
+        }
+        pair_sync(bar);
+        bool anym = true;  // the speculative path holds a match (V2: not tracked)
+        const uint64_t cm = ((uint64_t)rc0 << 32) | rc1;
+        if (MODE == kModeDumpMatch) {
+            // every candidate position through the production walk machine (a2)
+            uint8_t *LD = reinterpret_cast<uint8_t *>(dbg) + 2 * (start + B0);
+            walk_spec<true, !SMALLW>(ucw, link, sm.cw, bnd, cm, ld, LD, ce, m, cst, W, F, s0, s1, half, lane, (int)g.sw,
+                            (int)g.tx, anym);
+            if (last) return;
+            tileT1c = B0 + T1;
+            continue;
+        }
+        const int spec_exit =
+            V2 ? v2_jump(ld, s0, s1) : walk_spec<false, !SMALLW>(ucw, link, sm.cw, bnd, cm, ld, nullptr, ce, m, cst, W, F, s0, s1, half, lane,
+                                         (int)g.sw, (int)g.tx, anym);
+        int exitp = TILED && s0 < T0 ? Eb : spec_exit;  // window-history lanes hand on the tile's entry
+        int cur = s0;
+        bool first = true;
+        volatile uint32_t *xf = sm.a.u.w.xfer;
+        // two barriers per round: exits and "changed" flags use slots alternating
+        // with the round's parity, so a slot is rewritten only two rounds later,
+        // after every read of it
+        int par = 0;
+    #pragma unroll 1
+        while (true) {
+            // entry of walk lane t64 = exit of lane t64 - 1 (warp 1 lane 0 reads
+            // warp 0 lane 31 through shared memory)
+            int entry = __shfl_up_sync(kFull, exitp, 1);
+            if (lane == 31) xf[2 * par + half] = (uint32_t)exitp;
+            pair_sync(bar);
+            if (lane == 0) entry = half ? (int)xf[2 * par + half - 1] : 0;
+            const bool chg = (!TILED || (s0 >= T0 && s0 < T1)) && entry != cur;
+            const bool any = __any_sync(kFull, chg);
+            if (lane == 0) xf[4 + 2 * par + half] = any;
+            pair_sync(bar);
+            bool go = false;
+    #pragma unroll
+            for (int k = 0; k < kWarpsPerChunk; k++) go |= xf[4 + 2 * par + k] != 0;
+            if (!go) break;
+            par ^= 1;
+            if (chg) {
+                exitp = V2 ? v2_jump(ld, entry, s1)
+                           : walk_fix<!SMALLW>(ucw, link, cm, ld, ce, cst, W, F, s0, s1, entry, spec_exit, first);
+                first = false;
+                cur = entry;
+            }
+        }
+
+        // TILED: the tile's exit (ucw is dead after the walks; read after the next barrier)
+        if (TILED && !last && t64 == (T1 - 1) / kWSeg) ucw[0] = (uint32_t)exitp;
+        if (MODE == kModeDumpTokens) {
+            uint32_t *tok = reinterpret_cast<uint32_t *>(dbg) + start + B0;
+            for (int p = s0; p < s1; p++) tok[p] = 0;
+            int p = cur;
+            while (p < s1) {
+                if (!is_cand(cm, p - s0)) {
+                    tok[p] = 1;
+                    p++;
+                } else {
+                    const uint32_t t = ld[sk2(p)];
+                    tok[p] = Memo<!SMALLW>::is_match(t) ? ((uint32_t)Memo<!SMALLW>::len(t) << 16) | (uint32_t)Memo<!SMALLW>::dist(t)
+                                                        : 1u;
+                    p += Memo<!SMALLW>::len(t);
+                }
+            }
+            if (last) return;
+            pair_sync(bar);
+            Ec = B0 + (int)ucw[0];
+            tileT1c = B0 + T1;
+            continue;
+        }
+        pair_sync(bar);  // link is dead: staging may overwrite it
+        if (TILED && !last) Ec = B0 + (int)ucw[0];
+
+        // ---------------- a4: bit-pack ----------------------------------------
+        // Each walk lane emits its path's tokens MSB-first into its own staging
+        // words starting at bit 0 (a token is up to 3 literals of a candidate-free
+        // run, an evaluated literal, or a match); after the scan of bit counts the
+        // staged words are shifted into place.
+        uint32_t *stage = reinterpret_cast<uint32_t *>(sm.a.link) + t64 * kStageWords;
+        int nbits = 0;
+        {
+            // Uniform position scan (no token jumps): every position >= the lane's
+            // true entry is either inside a path match (covered) or a path token
+            // start; a token start's memoised ld[] is its token whichever walk
+            // wrote it, and is 0 for candidate-free positions (literals).  Each
+            // position emits 0, 9 or 17 bits.
+            uint64_t acc = 0;
+            int nacc = 0;
+            uint32_t *sp = stage;  // next staging word
+            int cov = cur;  // positions < cov are covered (by the previous lane or a match)
+            const int so = (s0 >> 7) << 2;
+            const uint32_t *ldw = reinterpret_cast<const uint32_t *>(ld + (so >> 1) + s0);  // 2 tokens / word
+            const uint32_t *cbw = reinterpret_cast<const uint32_t *>(cb + so + s0);         // 4 bytes / word
+            const int ng = (s1 - s0 + 3) >> 2;
+            // append pn (<= 26) bits; acc keeps < 32 pending bits between calls
+            auto put = [&](uint32_t pv, int pn) {
+                acc = (acc << pn) | pv;
+                nacc += pn;
+                if (nacc >= 32) {
+                    nacc -= 32;
+                    *sp++ = (uint32_t)(acc >> nacc);
                 }
             };
-            const int ngf = (s1 - s0) >> 2;  // full groups
-            int i = max(0, (cov - s0) >> 2);
-#pragma unroll 1
-            for (; i < ngf; i = max(i + 1, (cov - s0) >> 2)) group(i, false);
-            if (i == ngf && ngf < ng) group(i, true);
-        }
-        const int nw = (int)(sp - stage);
-        nbits = 32 * nw + nacc;
-        if (nacc > 0) *sp = (uint32_t)(acc << (32 - nacc));
-    }
-    // exclusive scan of bit counts over the 64 walk lanes
-    int incl = nbits;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const int y = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl += y;
-    }
-    if (lane == 31) xf[half] = (uint32_t)incl;
-    pair_sync(bar);
-    int before = 0, total = 0;
-#pragma unroll
-    for (int k = 0; k < kWarpsPerChunk; k++) {
-        const int v = (int)xf[k];
-        before += k < half ? v : 0;
-        total += v;
-    }
-    incl += before;
-    int excl = incl - nbits;
-    const uint64_t stride = bucket_stride(g.S);
-    const int kk = (m + (int)g.S - 1) / (int)g.S;  // chunks in this pair
-    int cbits = total, cword = 0;                  // this lane's chunk: total bits, first payload word
-    if (PACK) {
-        // packed chunks: a chunk's lanes are lpc consecutive lanes of one warp;
-        // bit offsets restart at each chunk, whose payload words start at its
-        // bucket offset in ow (the same layout as the buckets in HBM)
-        const int lpc = (int)g.S / kWSeg;
-        const int first = lane & ~(lpc - 1);
-        const int cbase = __shfl_sync(kFull, excl, first);
-        cbits = __shfl_sync(kFull, excl + nbits, first + lpc - 1) - cbase;
-        excl -= cbase;
-        cword = (t64 / lpc) * (int)(stride / 4);
-    }
-    const int nwords = PACK ? kk * (int)(stride / 4) : ((total + 31) >> 5) + 1;
-    uint32_t *ow = reinterpret_cast<uint32_t *>(ld);  // ld is dead: payload words
-#pragma unroll 4
-    for (int i = t64; i < nwords; i += kWalkLanes) ow[i] = 0;
-    pair_sync(bar);
-    {
-        // shift the lane's staged words to bit offset excl; output words shared
-        // with the neighbouring lanes (first, last, spill) are OR-ed atomically
-        const int sh = excl & 31;
-        const int base = cword + (excl >> 5);
-        const int nsw = (nbits + 31) >> 5;
-        if (nsw) {
-            // word i of the output = bits of staged words i-1, i shifted by sh
-            // (funnel shift: sh = 0 gives the word itself); the first and last
-            // (and the spill word) are shared with neighbours
-            uint32_t prev = stage[0];
-            atomicOr(&ow[base], prev >> sh);
-#pragma unroll 1
-            for (int i = 1; i < nsw - 1; i++) {
-                const uint32_t v = stage[i];
-                ow[base + i] = __funnelshift_r(v, prev, sh);
-                prev = v;
+            if (__all_sync(kFull, !anym && cur == s0 && s1 - s0 == kWSeg)) {
+                // every lane of the warp walks its whole segment from its start
+                // and found no match: 64 literals each (incompressible data),
+                // emitted branch-free in 18-bit pairs (bit positions static)
+    #pragma unroll
+                for (int i = 0; i < kWSeg / 4; i++) {
+                    const uint32_t bytes = cbw[i];
+                    put(((bytes & 0xFFu) << 9) | ((bytes >> 8) & 0xFFu), 18);
+                    put((((bytes >> 16) & 0xFFu) << 9) | (bytes >> 24), 18);
+                }
+            } else {
+                // groups wholly inside a match are skipped.  Positions are
+                // combined in pairs in 32 bits first: a pair is at most a literal
+                // and a match (26 bits), since a match covers the next position.
+                // Only a chunk's last lane can have a partial last group: full
+                // groups skip the segment-end test.
+                auto group = [&](int i, bool chk) {
+                    const uint32_t bytes = cbw[i];
+                    const uint32_t t01 = ldw[2 * i], t23 = ldw[2 * i + 1];
+                    uint32_t pv = 0;
+                    int pn = 0;
+    #pragma unroll
+                    for (int j = 0; j < 4; j++) {
+                        const int p = s0 + 4 * i + j;
+                        const uint32_t t = (j < 2 ? t01 : t23) >> (16 * (j & 1)) & 0xFFFFu;
+                        const bool on = p >= cov && (!chk || p < s1);
+                        const bool mt = on && Memo<!SMALLW>::is_match(t);
+                        const int nb = mt ? 17 : (on ? 9 : 0);
+                        const uint32_t val = mt ? Memo<!SMALLW>::code(t) : (on ? (bytes >> (8 * j)) & 0xFFu : 0u);  // 1|D-1|L-3
+                        cov = mt ? p + Memo<!SMALLW>::len(t) : cov;
+                        pv = (pv << nb) | val;
+                        pn += nb;
+                        if (j & 1) {
+                            put(pv, pn);
+                            pv = 0;
+                            pn = 0;
+                        }
+                    }
+                };
+                const int ngf = (s1 - s0) >> 2;  // full groups
+                int i = max(0, (cov - s0) >> 2);
+    #pragma unroll 1
+                for (; i < ngf; i = max(i + 1, (cov - s0) >> 2)) group(i, false);
+                if (i == ngf && ngf < ng) group(i, true);
             }
-            if (nsw > 1) {
-                const uint32_t v = stage[nsw - 1];
-                atomicOr(&ow[base + nsw - 1], __funnelshift_r(v, prev, sh));
-                prev = v;
-            }
-            const uint32_t o = sh ? prev << (32 - sh) : 0u;
-            if (o) atomicOr(&ow[base + nsw], o);
+            const int nw = (int)(sp - stage);
+            nbits = 32 * nw + nacc;
+            if (nacc > 0) *sp = (uint32_t)(acc << (32 - nacc));
         }
-    }
-    pair_sync(bar);
+        // exclusive scan of bit counts over the 64 walk lanes
+        int incl = nbits;
+    #pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(kFull, incl, o);
+            if (lane >= o) incl += y;
+        }
+        if (lane == 31) xf[half] = (uint32_t)incl;
+        pair_sync(bar);
+        int before = 0, total = 0;
+    #pragma unroll
+        for (int k = 0; k < kWarpsPerChunk; k++) {
+            const int v = (int)xf[k];
+            before += k < half ? v : 0;
+            total += v;
+        }
+        incl += before;
+        int excl = incl - nbits;
+        const int cb0 = TILED ? (boff & 127) : 0;  // TILED: bits of the carried partial unit come first
+        excl += cb0;
+        total += cb0;
+        const uint64_t stride = bucket_stride(g.S);
+        const int kk = (m + (int)g.S - 1) / (int)g.S;  // chunks in this pair
+        int cbits = total, cword = 0;                  // this lane's chunk: total bits, first payload word
+        if (PACK) {
+            // packed chunks: a chunk's lanes are lpc consecutive lanes of one warp;
+            // bit offsets restart at each chunk, whose payload words start at its
+            // bucket offset in ow (the same layout as the buckets in HBM)
+            const int lpc = (int)g.S / kWSeg;
+            const int first = lane & ~(lpc - 1);
+            const int cbase = __shfl_sync(kFull, excl, first);
+            cbits = __shfl_sync(kFull, excl + nbits, first + lpc - 1) - cbase;
+            excl -= cbase;
+            cword = (t64 / lpc) * (int)(stride / 4);
+        }
+        // (TILED: every word of the last, partial 16-byte unit, which is carried)
+        const int nwords = PACK ? kk * (int)(stride / 4) : (TILED ? 4 * ((total + 127) >> 7) + 4 : ((total + 31) >> 5) + 1);
+        uint32_t *ow = reinterpret_cast<uint32_t *>(ld);  // ld is dead: payload words
+    #pragma unroll 4
+        for (int i = t64; i < nwords; i += kWalkLanes)
+            ow[i] = TILED && i < 4 ? (i == 0 ? cy0 : i == 1 ? cy1 : i == 2 ? cy2 : cy3) : 0u;
+        pair_sync(bar);
+        {
+            // shift the lane's staged words to bit offset excl; output words shared
+            // with the neighbouring lanes (first, last, spill) are OR-ed atomically
+            const int sh = excl & 31;
+            const int base = cword + (excl >> 5);
+            const int nsw = (nbits + 31) >> 5;
+            if (nsw) {
+                // word i of the output = bits of staged words i-1, i shifted by sh
+                // (funnel shift: sh = 0 gives the word itself); the first and last
+                // (and the spill word) are shared with neighbours
+                uint32_t prev = stage[0];
+                atomicOr(&ow[base], prev >> sh);
+    #pragma unroll 1
+                for (int i = 1; i < nsw - 1; i++) {
+                    const uint32_t v = stage[i];
+                    ow[base + i] = __funnelshift_r(v, prev, sh);
+                    prev = v;
+                }
+                if (nsw > 1) {
+                    const uint32_t v = stage[nsw - 1];
+                    atomicOr(&ow[base + nsw - 1], __funnelshift_r(v, prev, sh));
+                    prev = v;
+                }
+                const uint32_t o = sh ? prev << (32 - sh) : 0u;
+                if (o) atomicOr(&ow[base + nsw], o);
+            }
+        }
+        pair_sync(bar);
 
-    // payload(s) -> bucket c.. (bytes in stream order: big-endian words); with
-    // packed chunks the kk buckets are contiguous in HBM as in ow
-    const int nbytes = (cbits + 7) >> 3;
-    uint4 *dst = reinterpret_cast<uint4 *>(bucket + c * stride);
-    const uint4 *o4 = reinterpret_cast<const uint4 *>(ow);
-    const int n16 = PACK ? kk * (int)(stride / 16) : (nbytes + 15) >> 4;
-    for (int i = t64; i < n16; i += kWalkLanes) {
-        uint4 v = o4[i];
-        v.x = __byte_perm(v.x, 0, 0x0123);
-        v.y = __byte_perm(v.y, 0, 0x0123);
-        v.z = __byte_perm(v.z, 0, 0x0123);
-        v.w = __byte_perm(v.w, 0, 0x0123);
-        dst[i] = v;
-    }
-    if (PACK) {
-        const int lpc = (int)g.S / kWSeg;
-        if ((t64 & (lpc - 1)) == 0 && t64 / lpc < kk) sizes[c + t64 / lpc] = (uint32_t)nbytes;
-    } else if (t64 == 0) {
-        sizes[c] = (uint32_t)nbytes;
-    }
+        // payload(s) -> bucket c.. (bytes in stream order: big-endian words); with
+        // packed chunks the kk buckets are contiguous in HBM as in ow
+        const int nbytes = (cbits + 7) >> 3;
+        uint4 *dst = reinterpret_cast<uint4 *>(bucket + c * stride) + (TILED ? boff >> 7 : 0);
+        const uint4 *o4 = reinterpret_cast<const uint4 *>(ow);
+        // TILED: a non-last tile writes its whole 16-byte units and carries the rest
+        const int n16 = PACK ? kk * (int)(stride / 16) : (TILED && !last ? total >> 7 : (nbytes + 15) >> 4);
+        if (TILED && !last) {
+            const uint32_t *cyw = ow + 4 * (total >> 7);
+            cy0 = cyw[0], cy1 = cyw[1], cy2 = cyw[2], cy3 = cyw[3];
+        }
+        for (int i = t64; i < n16; i += kWalkLanes) {
+            uint4 v = o4[i];
+            v.x = __byte_perm(v.x, 0, 0x0123);
+            v.y = __byte_perm(v.y, 0, 0x0123);
+            v.z = __byte_perm(v.z, 0, 0x0123);
+            v.w = __byte_perm(v.w, 0, 0x0123);
+            dst[i] = v;
+        }
+        if (PACK) {
+            const int lpc = (int)g.S / kWSeg;
+            if ((t64 & (lpc - 1)) == 0 && t64 / lpc < kk) sizes[c + t64 / lpc] = (uint32_t)nbytes;
+        } else if (t64 == 0 && last) {
+            sizes[c] = TILED ? (uint32_t)(((boff & ~127) + total + 7) >> 3) : (uint32_t)nbytes;
+        }
+        if (last) break;
+        boff = (boff & ~127) + total;
+        tileT1c = B0 + T1;
+    }  // tiles
 }
 
-template <int MODE, bool SMALLW, bool V2, bool PACK>
+template <int MODE, bool SMALLW, bool V2, bool PACK, bool TILED = false>
 cudaError_t launch_mode(const uint8_t *in, uint64_t n, Geometry g, uint8_t *bucket,
                         uint32_t *sizes, void *dbg, cudaStream_t st) {
     const uint64_t C = (n + g.S - 1) / g.S;
     if (C == 0) return cudaSuccess;
     const size_t smem = sizeof(WarpSmem) * kChunksPerCta;
     static std::atomic<uint64_t> attr_devs{0};  // per device (the opt-in is per device context)
-    cudaError_t e = set_smem_attr_once(chunk_kernel<MODE, SMALLW, V2, PACK>, (int)smem, attr_devs);
+    cudaError_t e = set_smem_attr_once(chunk_kernel<MODE, SMALLW, V2, PACK, TILED>, (int)smem, attr_devs);
     if (e != cudaSuccess) return e;
     const uint64_t pairs = (C + g.K - 1) / g.K;
     const uint64_t blocks = (pairs + kChunksPerCta - 1) / kChunksPerCta;
-    chunk_kernel<MODE, SMALLW, V2, PACK><<<(unsigned)blocks, kChunksPerCta * kWalkLanes, smem, st>>>(in, n, g, bucket,
+    chunk_kernel<MODE, SMALLW, V2, PACK, TILED><<<(unsigned)blocks, kChunksPerCta * kWalkLanes, smem, st>>>(in, n, g, bucket,
                                                                                             sizes, dbg);
     count_launch();
     return cudaGetLastError();
@@ -1068,6 +1115,9 @@ template <int MODE>
 cudaError_t launch_w(const uint8_t *in, uint64_t n, Geometry g, uint8_t *bucket, uint32_t *sizes,
                      void *dbg, cudaStream_t st) {
     const bool pack = g.K > 1;
+    if (g.S > (uint32_t)kChunkMax)  // large chunks (version 0 only): compressed in tiles
+        return g.W <= 128 ? launch_mode<MODE, true, false, false, true>(in, n, g, bucket, sizes, dbg, st)
+                          : launch_mode<MODE, false, false, false, true>(in, n, g, bucket, sizes, dbg, st);
     if (g.V == 2)
         return pack ? launch_mode<MODE, false, true, true>(in, n, g, bucket, sizes, dbg, st)
                     : launch_mode<MODE, false, true, false>(in, n, g, bucket, sizes, dbg, st);

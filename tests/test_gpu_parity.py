@@ -244,7 +244,7 @@ def test_buffer_too_small_and_invalid(env):
         culzss.compress(x, culzss.Params.make(MIN=2))
     assert e.value.status == culzss.ERR_INVALID_ARG
     with pytest.raises(culzss.CulzssError) as e:
-        culzss.compress(x, culzss.Params.make(S=8192))
+        culzss.compress(x, culzss.Params.make(S=65537))  # S <= 64 KiB (tiled above 4 KiB)
     assert e.value.status == culzss.ERR_UNSUPPORTED
 
 
