@@ -16,6 +16,8 @@
 #include <vector>
 #include <algorithm>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "../../include/culzss.h"
 #include "culzss_internal.h"
 
@@ -55,6 +57,13 @@ void lib_init() {
         cudaGetLastError();
     });
 }
+
+// NVTX range around each ABI call (visible in nsys / ncu --nvtx timelines;
+// a no-op unless a tool is attached)
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 
 struct LibLoad {
     LibLoad() { /* device detection is lazy: CUDA may not be usable at dlopen time */ }
@@ -321,6 +330,7 @@ culzss_status culzss_write_header(void *out, size_t n_total, const culzss_params
 
 culzss_status culzss_compress(const void *in, size_t n, void *out, size_t *out_n,
                               const culzss_params *p, culzss_stream_t stream) {
+    NvtxRange nvtx_("culzss_compress");
     lib_init();
     if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
     if (!out_n) return CULZSS_ERR_INVALID_ARG;
@@ -372,6 +382,7 @@ culzss_status culzss_compress(const void *in, size_t n, void *out, size_t *out_n
 culzss_status culzss_compress_chunks(const void *in_slice, size_t slice_n, void *payload,
                                      size_t *payload_n, uint32_t *chunk_sizes,
                                      const culzss_params *p, culzss_stream_t stream) {
+    NvtxRange nvtx_("culzss_compress_chunks");
     lib_init();
     if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
     if (!payload_n) return CULZSS_ERR_INVALID_ARG;
@@ -418,6 +429,7 @@ culzss_status culzss_compress_chunks(const void *in_slice, size_t slice_n, void 
 culzss_status culzss_compress_chunks_async(const void *in_slice, size_t slice_n, void *payload,
                                            size_t payload_cap, uint32_t *chunk_sizes, uint64_t *dev_total,
                                            const culzss_params *p, culzss_stream_t stream) {
+    NvtxRange nvtx_("culzss_compress_chunks_async");
     lib_init();
     if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
     Geometry g;
@@ -493,6 +505,7 @@ thread_local HostPipe t_pipe_dev[kMaxDevices];  // streams/events of the current
 
 culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host, size_t *out_n,
                                    const culzss_params *p, culzss_stream_t stream) {
+    NvtxRange nvtx_("culzss_compress_host");
     lib_init();
     if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
     if (!out_n || (n && !in_host) || !out_host) return CULZSS_ERR_INVALID_ARG;
@@ -711,6 +724,7 @@ static culzss_status decompress_core(const uint8_t *payload, uint64_t pay_len, c
 
 culzss_status culzss_decompress(const void *in, size_t in_n, void *out, size_t *out_n,
                                 const culzss_params *, culzss_stream_t stream) {
+    NvtxRange nvtx_("culzss_decompress");
     lib_init();
     if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
     if (!out_n || !is_device_ptr(in)) return CULZSS_ERR_INVALID_ARG;
@@ -739,6 +753,7 @@ culzss_status culzss_decompress(const void *in, size_t in_n, void *out, size_t *
 culzss_status culzss_decompress_chunks(const void *payload, size_t payload_n, const uint32_t *chunk_sizes,
                                        size_t slice_n, void *out, const culzss_params *p,
                                        culzss_stream_t stream) {
+    NvtxRange nvtx_("culzss_decompress_chunks");
     lib_init();
     if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
     Geometry g;
@@ -762,6 +777,7 @@ culzss_status culzss_decompress_chunks(const void *payload, size_t payload_n, co
 // the single final sync.
 culzss_status culzss_decompress_host(const void *in_host, size_t in_n, void *out_host, size_t *out_n,
                                      const culzss_params *, culzss_stream_t stream) {
+    NvtxRange nvtx_("culzss_decompress_host");
     lib_init();
     if (g_device_count <= 0) return CULZSS_ERR_NO_DEVICE;
     if (!out_n || !in_host || !out_host) return CULZSS_ERR_INVALID_ARG;

@@ -13,8 +13,9 @@
 //   a4  bit-pack  flag 0 + byte | flag 1 + (D-1) + (L-3), MSB first, zero pad
 //                 (PAPER.md:1@4785, @23049-23282; readings R9-R11)
 //
-// B200 design: a PAIR of warps per 4 KiB chunk (three pairs per
-// 192-thread CTA, three CTAs per SM), everything in shared memory:
+// B200 design: a PAIR of warps per 4 KiB chunk, one chunk per
+// 64-thread CTA, nine CTAs per SM (24.8 KB of shared memory each: a chunk's
+// memory is released as soon as it finishes), everything in shared memory:
 //   * Chain build (a2, part 1; warp 0).  Lane l owns the 128-position build
 //     segment [128l, 128l + 128) and a private 512-bucket u8 hash table
 //     ([lane][bucket]); it inserts the W positions before its segment, then
@@ -27,20 +28,25 @@
 //   * Lazy greedy walk (a2 part 2 + a3; both warps).  Walk lane t (0..63) runs
 //     the greedy parse over the 64-position segment [64t, 64t + 64) from its
 //     start, evaluating L/D only where the parse lands -- the V1 "jump over"
-//     saving (PAPER.md:1@32329 §V).  The walk is one flat state machine per
+//     saving (PAPER.md:1@32329 §V).  Machine 1 is a flat state machine per
 //     lane: every iteration is one 8-byte compare (big-endian words of an
 //     unskewed chunk copy, equal leading bytes by a 64-bit clz) of one
 //     candidate -- an 8-byte reject test at [bestL-7, bestL] once bestL >= 8,
 //     else an LCP step -- and positions without a candidate are skipped with a
-//     64-bit mask.  Fix-up rounds then hand each lane its true entry (the
-//     previous lane's exit); a lane whose entry moved re-walks only until it
-//     meets its earlier path.  The result is exactly the serial greedy parse.
+//     64-bit mask.  A warp one of whose lanes spends 16 iterations on one token
+//     switches to machine 2, the same walk with two exact prunes (run skip,
+//     chain switch; see walk_spec).  Fix-up rounds then hand each lane its true
+//     entry (the previous lane's exit); a lane whose entry moved re-walks only
+//     until it meets its earlier path.  The result is exactly the serial
+//     greedy parse.
 //   * Bit-pack (a4): each lane emits its path's tokens (positions combined in
 //     32-bit pairs), a 64-lane scan of bit counts places them, edge words are
 //     OR-ed, and the payload goes to the chunk's bucket with 16-byte stores.
 //   * params.version = 2 replaces the build and walk by the paper's V2 search
 //     (every position, every offset, warp argmax); chunks of S = 64..2048 are
-//     packed 4096 / S to a pair (PACK).
+//     packed 4096 / S to a pair (PACK); chunks of S > 4096 are compressed in
+//     4096-position tiles (TILED); W = 256 adds d = 256 as one extra candidate
+//     (the u8 links hold <= 255).
 
 #include "culzss_internal.h"
 
