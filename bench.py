@@ -111,7 +111,7 @@ def load_int_peak():
     LOP3 rate measured by tools/micro/int_peak.cu -- live on this GPU when the
     binary is built, else the committed B200 measurement."""
     exe = os.path.join(ROOT, "tools", "micro", "int_peak")
-    if os.path.exists(exe):
+    if os.path.exists(exe) and not os.environ.get("CULZSS_BENCH_NO_LIVE_PEAK"):  # (set under a profiler)
         try:
             r = subprocess.run([exe], capture_output=True, text=True, timeout=60)
             d = json.loads(r.stdout.strip().splitlines()[-1])

@@ -70,6 +70,8 @@ def launches(path):
         if r.get("Metric Name") != "gpu__time_duration.sum":
             continue
         name = r["Kernel Name"].split("(")[0].replace("void ", "")
+        if name.startswith("k_int"):  # bench.py's integer-peak microbenchmark (a child process), not the step
+            continue
         v = float(r["Metric Value"].replace(",", ""))
         unit = r.get("Metric Unit", "")
         scale = {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0, "msecond": 1e3,
