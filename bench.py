@@ -106,14 +106,15 @@ def rank_input(cfg: str, rank: int, world: int, scaling: str = "strong") -> np.n
     return datagen.generate_range(datagen.CONFIGS[cfg]["kind"], n, seed, b0, b1)
 
 
-def load_int_peak():
+def load_int_peak(device: int = 0, live: bool = True):
     """Integer-pipe peak for the compare term: the ALU-pipe
-    LOP3 rate measured by tools/micro/int_peak.cu -- live on this GPU when the
-    binary is built, else the committed B200 measurement."""
+    LOP3 rate measured by tools/micro/int_peak.cu -- live on this rank's GPU
+    when the binary is built, else the committed B200 measurement (also when
+    several ranks share one GPU, or under a profiler)."""
     exe = os.path.join(ROOT, "tools", "micro", "int_peak")
-    if os.path.exists(exe) and not os.environ.get("CULZSS_BENCH_NO_LIVE_PEAK"):  # (set under a profiler)
+    if live and os.path.exists(exe) and not os.environ.get("CULZSS_BENCH_NO_LIVE_PEAK"):
         try:
-            r = subprocess.run([exe], capture_output=True, text=True, timeout=60)
+            r = subprocess.run([exe, str(device)], capture_output=True, text=True, timeout=60)
             d = json.loads(r.stdout.strip().splitlines()[-1])
             if r.returncode == 0:
                 return d, "measured live on this GPU (tools/micro/int_peak.cu, LOP3 / ALU pipe)"
@@ -506,7 +507,7 @@ def main():
     # searches only where the greedy parse lands, through hash chains with
     # exact prunes, so it can beat the compare term; HBM is the hard floor.
     hbm_peak, sm_max_mhz, peak_kind = load_peaks()
-    ip, ip_src = load_int_peak()
+    ip, ip_src = load_int_peak(local, live=backend == "nccl" or world == 1)
     int_peak_tops = float(ip["lop3_tops"])
     pay_bytes = (out_n - 32 - 4 * C) if world == 1 else placed.payload_bytes
     ck = statistics.mean(chunk_ms)

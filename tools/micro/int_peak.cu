@@ -5,7 +5,7 @@
 // are LOP3 / IADD3, which issue only on the ALU pipe.
 //
 //   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o int_peak tools/micro/int_peak.cu
-//   ./int_peak > profiles/int_peak.json       (one JSON object)
+//   ./int_peak [device] > profiles/int_peak.json       (one JSON object)
 //
 // Each thread runs 8 independent accumulator chains through an unrolled
 // loop of inline-PTX instructions (lop3.b32 / add of three operands that
@@ -13,6 +13,7 @@
 // (8 chains x 16 warps per SMSP).  Check the SASS with
 //   cuobjdump -sass int_peak | grep -c LOP3    (etc.)
 #include <cstdio>
+#include <cstdlib>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -73,9 +74,9 @@ double run(int sms, uint32_t *d, cudaEvent_t e0, cudaEvent_t e1, int blocks_per_
     return ops / (best * 1e-3) / 1e12;  // Tops/s
 }
 
-int main() {
-    int dev = 0, sms = 0, clk_khz = 0;
-    cudaGetDevice(&dev);
+int main(int argc, char **argv) {
+    int dev = argc > 1 ? atoi(argv[1]) : 0, sms = 0, clk_khz = 0;  // device ordinal (bench.py passes its rank's)
+    cudaSetDevice(dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaDeviceGetAttribute(&clk_khz, cudaDevAttrClockRate, dev);
     cudaDeviceProp prop;
