@@ -56,6 +56,7 @@ namespace {
 constexpr uint32_t kFull = 0xffffffffu;
 constexpr uint32_t kTabBias = 0x1000;   // table entry = position + bias; 0 = empty
 constexpr uint32_t kHashMul = 0x9E3779B1u << 8;
+constexpr int kSparseLinks = 24;  // candidate-mask filter: at most this many linked positions per lane of the warp
 // Memoised token encoding in ld[] (u16).  W <= 128: 0 = not evaluated,
 // 2 = literal, (D << 8) | (L - 3) = match (>= 0x100; L - 3 fits 8 bits for
 // F <= 258).  W > 128 (BW; W = 256 needs D = 256): 0 = not evaluated,
@@ -815,6 +816,7 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         }
         // candidate mask: bit i = position s0 + i (< s1) has a chain link
         uint32_t rc0 = 0, rc1 = 0;
+        uint32_t h[2] = {0, 0};
         if (V2) {
             // every position holds its evaluated token
             const int r = max(s1 - s0, 0);
@@ -822,7 +824,6 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
             rc1 = r <= 32 ? 0u : (r >= 64 ? 0xFFFFFFFFu : ~(0xFFFFFFFFu >> (r - 32)));
         } else if (s0 < s1) {
             const int so = (s0 >> 7) << 2;  // constant skew inside the segment
-            uint32_t h[2] = {0, 0};
     #pragma unroll
             for (int w = 0; w < kWSeg / 4; w++) {
                 const uint32_t lw = *reinterpret_cast<const uint32_t *>(link + so + s0 + 4 * w);
@@ -842,6 +843,28 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
                 h[0] &= r >= 32 ? 0xFFFFFFFFu : (1u << r) - 1;
                 h[1] &= r <= 32 ? 0u : (1u << (r - 32)) - 1;
             }
+        }
+        // a position whose chain is one hash collision and nothing more has
+        // no candidate at all: a literal, never evaluated.  Checked where
+        // every lane of the warp has sparse links (incompressible data,
+        // whose candidates are nearly all collisions; on text the chains
+        // continue and the check would only cost)
+        if (!V2 && SMALLW && __all_sync(kFull, __popc(h[0]) + __popc(h[1]) <= kSparseLinks)) {
+#pragma unroll
+            for (int hw = 0; hw < 2; hw++) {
+                uint32_t keep = h[hw];
+#pragma unroll 1
+                for (uint32_t b = h[hw]; b; b &= b - 1) {
+                    const int p = s0 + 32 * hw + __ffs(b) - 1;
+                    const int d = link[sk(p)];
+                    const int l2 = link[sk(p - d)];
+                    const bool eq3 = ((load4(sm.cw, p) ^ load4(sm.cw, p - d)) & 0xFFFFFFu) == 0;
+                    if (!eq3 && (l2 == 0 || d + l2 > W)) keep &= ~(1u << (p - s0 - 32 * hw));
+                }
+                h[hw] = keep;
+            }
+        }
+        if (!V2) {
             rc0 = __brev(h[0]);
             rc1 = __brev(h[1]);
         }
