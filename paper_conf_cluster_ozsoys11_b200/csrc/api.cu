@@ -520,11 +520,15 @@ culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host
         return CULZSS_ERR_BUFFER_TOO_SMALL;
     }
     cudaStream_t st = (cudaStream_t)stream;
-    static const uint64_t group_bytes = [] {  // CULZSS_GROUP_KB: pipeline tuning knob
+    // group size: 8 MiB, 16 MiB from 512 MiB of input on (fewer per-group host
+    // waits; B200: c2 128 MiB 44.8 GB/s at 8 MiB vs 38.4 at 16; c3 1 GiB 51.2 vs
+    // 52.5).  CULZSS_GROUP_KB overrides (pipeline tuning knob)
+    static const uint64_t group_env = [] {
         const char *e = getenv("CULZSS_GROUP_KB");
         const long v = e ? atol(e) : 0;
-        return v > 0 ? (uint64_t)v << 10 : (8ull << 20);
+        return v > 0 ? (uint64_t)v << 10 : 0ull;
     }();
+    const uint64_t group_bytes = group_env ? group_env : (n >= (512ull << 20) ? 16ull << 20 : 8ull << 20);
     const uint64_t gc = std::max<uint64_t>(1, group_bytes / g.S);  // chunks per group
     const uint64_t G = (C + gc - 1) / gc;
     if (G <= 1) {  // one group: no overlap to gain
@@ -807,11 +811,12 @@ culzss_status culzss_decompress_host(const void *in_host, size_t in_n, void *out
     const uint64_t pay_len = in_n - 32 - 4 * C;
     if (off[C] != pay_len) return CULZSS_ERR_CORRUPT;
     cudaStream_t st = (cudaStream_t)stream;
-    static const uint64_t dgroup_bytes = [] {  // CULZSS_DGROUP_KB: decode group size (output bytes)
+    static const uint64_t dgroup_env = [] {  // CULZSS_DGROUP_KB: decode group size (output bytes)
         const char *e = getenv("CULZSS_DGROUP_KB");
         const long v = e ? atol(e) : 0;
-        return v > 0 ? (uint64_t)v << 10 : (8ull << 20);
+        return v > 0 ? (uint64_t)v << 10 : 0ull;
     }();
+    const uint64_t dgroup_bytes = dgroup_env ? dgroup_env : (n >= (512ull << 20) ? 16ull << 20 : 8ull << 20);
     const uint64_t gc = std::max<uint64_t>(1, dgroup_bytes / g.S);  // chunks per group
     const uint64_t G = (C + gc - 1) / gc;
     HostPipe &hp = t_pipe_dev[cur_device()];
