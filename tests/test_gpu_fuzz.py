@@ -27,10 +27,17 @@ def test_random_cases(env, seed):
     for _ in range(25):
         kind = str(rng.choice(datagen.GENERATORS))
         n = int(rng.integers(1, 200_000))
-        S = int(rng.choice([64, 128, 256, 512, 1024, 2048, 4096, int(rng.integers(1, 4097))]))
-        W = int(rng.integers(1, 256))
+        S = int(rng.choice([64, 128, 256, 512, 1024, 2048, 4096, int(rng.integers(1, 4097)),
+                            int(rng.integers(4097, 65537))]))
+        W = int(rng.integers(1, 257))
         F = int(rng.integers(3, 259))
         version = int(rng.choice([0, 0, 2]))
+        # the GPU path's limits: version 2 up to S = 4096 and W = 255;
+        # W = 256 needs F <= 256
+        if version == 2 and (S > 4096 or W == 256):
+            version = 0
+        if W == 256:
+            F = min(F, 256)
         x = datagen.generate(kind, n, seed=int(rng.integers(0, 1 << 30)))
         p = culzss.Params.make(S=S, W=W, F=F, version=version)
         s = culzss.compress(dev(torch, x), p)
