@@ -469,9 +469,9 @@ culzss_status culzss_compress_chunks_async(const void *in_slice, size_t slice_n,
 namespace {
 constexpr int kPipeStreams = 3;
 struct HostPipe {
-    cudaStream_t cs[kPipeStreams] = {}, ds = {};
+    cudaStream_t cs[kPipeStreams] = {}, ds = {}, hs = {};  // compute streams, D2H stream, H2D stream
     cudaEvent_t ev_in = {};
-    std::vector<cudaEvent_t> ev;
+    std::vector<cudaEvent_t> ev, evh;  // per group: kernels + table copy done; its H2D done
     uint64_t *htot = nullptr;  // mapped pinned: the scan kernel writes group totals here
     uint64_t *dtot = nullptr;  // its device alias
     size_t htot_n = 0;
@@ -481,14 +481,17 @@ struct HostPipe {
             for (auto &c : cs)
                 if (cudaStreamCreateWithFlags(&c, cudaStreamNonBlocking) != cudaSuccess) return false;
             if (cudaStreamCreateWithFlags(&ds, cudaStreamNonBlocking) != cudaSuccess ||
+                cudaStreamCreateWithFlags(&hs, cudaStreamNonBlocking) != cudaSuccess ||
                 cudaEventCreateWithFlags(&ev_in, cudaEventDisableTiming) != cudaSuccess)
                 return false;
             ok = true;
         }
         while (ev.size() < groups) {
-            cudaEvent_t e;
+            cudaEvent_t e, f;
             if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) return false;
+            if (cudaEventCreateWithFlags(&f, cudaEventDisableTiming) != cudaSuccess) return false;
             ev.push_back(e);
+            evh.push_back(f);
         }
         if (htot_n < groups) {
             if (htot) cudaFreeHost(htot);
@@ -570,6 +573,7 @@ culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host
             if (done) return;
             for (auto cs : hp.cs) cudaStreamSynchronize(cs);
             cudaStreamSynchronize(hp.ds);
+            cudaStreamSynchronize(hp.hs);
             cudaGetLastError();
         }
     } drain{hp};
@@ -579,6 +583,15 @@ culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host
     CK(cudaEventRecord(hp.ev_in, st));  // the workspace and header exist
     for (auto cs : hp.cs) CK(cudaStreamWaitEvent(cs, hp.ev_in, 0));
     CK(cudaStreamWaitEvent(hp.ds, hp.ev_in, 0));
+    CK(cudaStreamWaitEvent(hp.hs, hp.ev_in, 0));
+    // every group's H2D up front, back to back on the H2D stream: the
+    // host->device copy engine never waits for the issue loop below
+    for (uint64_t k = 0; k < G; k++) {
+        const uint64_t c0 = k * gc, c1 = std::min(C, c0 + gc);
+        const uint64_t b0 = c0 * g.S, nb = std::min<uint64_t>(n, c1 * g.S) - b0;
+        CK(cudaMemcpyAsync(din + b0, hin + b0, nb, cudaMemcpyHostToDevice, hp.hs));
+        CK(cudaEventRecord(hp.evh[k], hp.hs));
+    }
     CK(cudaMemcpyAsync(hout, dht, 32, cudaMemcpyDeviceToHost, hp.ds));
     uint64_t base = 0;  // payload bytes of the groups whose D2H is issued
     auto issue_payload = [&](uint64_t k) -> culzss_status {
@@ -596,7 +609,7 @@ culzss_status culzss_compress_host(const void *in_host, size_t n, void *out_host
         cudaStream_t cs = hp.cs[k % kPipeStreams];
         const uint64_t c0 = k * gc, c1 = std::min(C, c0 + gc);
         const uint64_t b0 = c0 * g.S, nb = std::min<uint64_t>(n, c1 * g.S) - b0;
-        CK(cudaMemcpyAsync(din + b0, hin + b0, nb, cudaMemcpyHostToDevice, cs));
+        CK(cudaStreamWaitEvent(cs, hp.evh[k], 0));
         s = compress_core(din + b0, nb, g, dstg + payload_bound(b0, g.S),
                           reinterpret_cast<uint32_t *>(dht + 32) + c0, nullptr, hp.dtot + k, cs,
                           dcore + (k % kPipeStreams) * core_bytes, false);  // no per-group profiling events in the issue loop
@@ -839,6 +852,7 @@ culzss_status culzss_decompress_host(const void *in_host, size_t in_n, void *out
             if (done) return;
             for (auto cs : hp.cs) cudaStreamSynchronize(cs);
             cudaStreamSynchronize(hp.ds);
+            cudaStreamSynchronize(hp.hs);
             cudaGetLastError();
         }
     } drain{hp};
@@ -848,14 +862,21 @@ culzss_status culzss_decompress_host(const void *in_host, size_t in_n, void *out
     CK(cudaEventRecord(hp.ev_in, st));  // the workspace exists and the error word is clear
     for (auto cs : hp.cs) CK(cudaStreamWaitEvent(cs, hp.ev_in, 0));
     CK(cudaStreamWaitEvent(hp.ds, hp.ev_in, 0));
+    CK(cudaStreamWaitEvent(hp.hs, hp.ev_in, 0));
+    // every group's H2D (table slice + payload) up front on the H2D stream
+    for (uint64_t k = 0; k < G; k++) {
+        const uint64_t c0 = k * gc, c1 = std::min(C, c0 + gc);
+        CK(cudaMemcpyAsync(dtab + 4 * c0, hin + 32 + 4 * c0, 4 * (c1 - c0), cudaMemcpyHostToDevice, hp.hs));
+        if (off[c1] > off[c0])
+            CK(cudaMemcpyAsync(dpay + off[c0], hin + 32 + 4 * C + off[c0], off[c1] - off[c0],
+                               cudaMemcpyHostToDevice, hp.hs));
+        CK(cudaEventRecord(hp.evh[k], hp.hs));
+    }
     for (uint64_t k = 0; k < G; k++) {
         cudaStream_t cs = hp.cs[k % kPipeStreams];
         const uint64_t c0 = k * gc, c1 = std::min(C, c0 + gc);
         const uint64_t b0 = c0 * g.S, nb = std::min<uint64_t>(n, c1 * g.S) - b0;
-        CK(cudaMemcpyAsync(dtab + 4 * c0, hin + 32 + 4 * c0, 4 * (c1 - c0), cudaMemcpyHostToDevice, cs));
-        if (off[c1] > off[c0])
-            CK(cudaMemcpyAsync(dpay + off[c0], hin + 32 + 4 * C + off[c0], off[c1] - off[c0],
-                               cudaMemcpyHostToDevice, cs));
+        CK(cudaStreamWaitEvent(cs, hp.evh[k], 0));
         s = decompress_enqueue(dpay + off[c0], off[c1] - off[c0], dtab + 4 * c0, c1 - c0, nb, g, dout + b0, cs, err,
                                false);
         if (s != CULZSS_OK) return s;
