@@ -3,7 +3,7 @@
 TAG=$1; cfg=${2:-c4_random_1g}
 cd "${GRAFT_REPO_ROOT:-$(dirname "$0")/..}"
 mkdir -p gpurun_out
-ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"walk_kernel|decode_kernel" -c 6 --csv \
+ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"classify_kernel|walk_kernel|decode_kernel|literal_kernel" -c 12 --csv \
     --log-file gpurun_out/declaunch_${cfg}_$TAG.csv python bench.py --config $cfg --steps 2 --warmup 1 --no-cpu-baseline \
     --no-e2e --no-versions --no-other-configs > /dev/null 2>&1
 python - gpurun_out/declaunch_${cfg}_$TAG.csv <<'PY'
