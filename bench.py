@@ -640,7 +640,7 @@ def main():
         line["decompress"] = {"value": n / (statistics.mean(cms) / 1000) / 1e9, "unit": "GB/s (output)",
                               "decode_kernel_ms": dk, "call_ms": statistics.mean(cms),
                               "roundtrip_exact": ok,
-                              "roofline": {"bound": "hbm", "kernels": "decoder kernels (walk + decode)",
+                              "roofline": {"bound": "hbm", "kernels": "decoder kernels (classify + literal + walk + decode)",
                                            "algorithmic_bytes": dec_bytes,
                                            "achieved": dec_bytes / (dk / 1000) / 1e9, "peak": hbm_peak,
                                            "unit": "GB/s", "frac": dec_bytes / (dk / 1000) / 1e9 / hbm_peak,
