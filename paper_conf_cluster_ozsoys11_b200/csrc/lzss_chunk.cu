@@ -545,49 +545,130 @@ __device__ int walk_fix(const uint32_t *__restrict__ u, const uint8_t *__restric
 // thread ... is responsible for one character of the uncoded lookahead
 // buffer" and searches the whole window buffer for it; "all the matches are
 // searched ... redundant ones are eliminated" @17800) as the north star's
-// warp-cooperative kernel: for EVERY position p of the chunk the warp
-// evaluates all window offsets at once, lane l taking d = l+1, l+33, l+65,
-// l+97 (l+129, ... for W > 128).  Each offset's run is measured with packed
-// 32-bit compares (XOR of 4 bytes; the first differing byte ends the run, a
-// fully equal word extends it 4 bytes at a time), and the warp's argmax is
-// one __reduce_max_sync over (L << 8) | (255 - (d - 1)): the largest L, ties
-// to the smallest d (reading R7).  L < 3 is a literal (R4).  The result is the
-// same (L, D) table the lazy walk evaluates on demand, so the greedy parse
-// and the bit-pack downstream are shared.  It executes the brute-force
-// compare count of the roofline's compare term.
-__device__ __forceinline__ uint32_t v2_run(const uint32_t *cw, int p, int d, uint32_t p0, int cap) {
-    const int q = p - d;
-    uint32_t x = load4(cw, q) ^ p0;
-    int k = 4;
-    // early out on the first differing byte; equal words extend the run
-    while (!x && k < cap) {
-        x = load4(cw, q + k) ^ load4(cw, p + k);
-        k += 4;
-    }
-    const int L = x ? k - 4 + ((__ffs(x) - 1) >> 3) : k;
-    return (uint32_t)min(L, cap);
+// warp-cooperative kernel: (L, D) of EVERY position over EVERY window offset.
+// Lane l owns the offsets d = l + 1 + 32k (k < K; K = 4 for W <= 128, 8
+// above); warp h sweeps half the chunk's positions from the top down, one
+// 32-bit word (4 positions) per step, with the diagonal run recurrence
+//     R_d(p) = (chunk[p] == chunk[p-d]) ? min(R_d(p+1) + 1, F) : 0,
+// whose equalities come from one packed 32-bit compare (XOR + exact
+// zero-byte test) of bytes p..p+3 against p-d..p-d+3 per offset -- the
+// compare count of the roofline's compare term, with no
+// data-dependent early-out loop.  R_d(p) <= m - p because the sweep starts
+// at the chunk end with R = 0 (and restarts at every packed chunk boundary);
+// pairs with d > p - chunk start or d > W never match.  The argmax over d is
+// one __reduce_max_sync per position over (L << 8) | (256 - d): the largest L,
+// ties to the smallest d (reading R7); L < 3 is a literal (R4).  The result is
+// the same (L, D) table the lazy walk evaluates on demand, so the greedy parse
+// and the bit-pack downstream are shared.
+//
+// bytes x..x+3 (little endian) of the unskewed chunk copy U (x >= 0)
+__device__ __forceinline__ uint32_t v2_bytes4(const uint32_t *__restrict__ U, int x) {
+    const uint32_t a = (uint32_t)x >> 2;
+    return __funnelshift_r(U[a], U[a + 1], (uint32_t)x << 3);  // the shift is taken mod 32
 }
 
-__device__ void v2_search_all(const uint32_t *cw, uint16_t *ld, int m, int W, int F, int half, int lane,
-                              int smask) {
-#pragma unroll 1
-    for (int p = half; p < m; p += kWarpsPerChunk) {
-        // window and lookahead stay inside p's chunk [p & ~smask, +S)
-        const int cap = min(F, min((p | smask) + 1, m) - p);
-        const int dmax = min(W, p & smask);
-        uint32_t best = 0;
-        if (cap >= 3) {
-            const uint32_t p0 = load4(cw, p);  // same word for every lane (broadcast)
-#pragma unroll 4
-            for (int d = lane + 1; d <= dmax; d += 32) {
-                const uint32_t L = v2_run(cw, p, d, p0, cap);
-                const uint32_t key = L >= 3 ? (L << 8) | (uint32_t)(256 - d) : 0u;
-                best = max(best, key);
+template <int K>
+__device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restrict__ ld, int m, int W, int F,
+                              int half, int lane, int smask) {
+    // warp 0: positions [0, M0), warp 1: [M0, m); M0 is a word boundary
+    const int M0 = ((m >> 1) + 3) & ~3;
+    const int r0 = half ? M0 : 0, r1 = half ? m : M0;
+    if (r0 >= r1) return;
+    int R[K];
+    uint32_t dead[K];  // 0x80808080: offset beyond W (never matches)
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        const int d = lane + 1 + 32 * k;
+        dead[k] = d <= W ? 0u : 0x80808080u;
+        // the run at r1 (the carry into the sweep): 0 at the chunk end or at a
+        // packed chunk boundary, else measured directly
+        int r = 0;
+        if (r1 < m && (r1 & smask) != 0 && d <= W && d <= (r1 & smask)) {
+            const int cap = min(F, min((r1 | smask) + 1, m) - r1);
+            while (r < cap) {
+                const uint32_t x = v2_bytes4(U, r1 + r) ^ v2_bytes4(U, r1 - d + r);
+                if (x) {
+                    r += (__ffs(x) - 1) >> 3;
+                    break;
+                }
+                r += 4;
             }
+            r = min(r, cap);
         }
-        best = __reduce_max_sync(kFull, best);
-        if (lane == 0) ld[sk2(p)] = best ? (uint16_t)Memo<true>::match((int)(256 - (best & 0xFF)), (int)(best >> 8))
-                                         : Memo<true>::kLit;
+        R[k] = r;
+    }
+    // One step: the 4 positions of word p0.  EDGE steps (the first W
+    // positions of a chunk, where d > p - chunk start, and the buffer's last,
+    // partial word) mask the invalid pairs; the others are straight-line: for
+    // offset d_k = lane + 1 + 32k the bytes p0 - d_k .. + 3 lie in the aligned
+    // words at byte offsets p0 - c4 - 32k and + 4 (c4 = d_0 rounded up to a
+    // multiple of 4), shifted by the same amount for every k.
+    const int c4 = (lane + 4) & ~3;
+    const uint32_t shq = 8u * (uint32_t)((-(lane + 1)) & 3);
+    const unsigned char *Ub = reinterpret_cast<const unsigned char *>(U);
+    auto step = [&](int p0, bool edge) {
+        const uint32_t P = U[p0 >> 2];
+        const int lowp = p0 & smask;               // position of p0 in its chunk
+        const bool bnd = ((p0 + 4) & smask) == 0;  // a chunk ends after this word: no carry
+        uint32_t best0 = 0, best1 = 0, best2 = 0, best3 = 0;
+        const unsigned char *qa = Ub + (p0 - c4);
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            const int d = lane + 1 + 32 * k;
+            uint32_t Q;
+            if (!edge) {
+                const uint32_t *w = reinterpret_cast<const uint32_t *>(qa - 32 * k);
+                Q = __funnelshift_r(w[0], w[1], shq);
+            } else {
+                // before the buffer start (-3 <= q < 0 holds valid bytes) the
+                // first word shifted into place
+                const int q = p0 - d;
+                Q = q >= 0 ? v2_bytes4(U, q) : v2_bytes4(U, 0) << (8 * min(-q, 3));
+            }
+            const uint32_t x = P ^ Q;
+            // bit 7 of byte j set iff byte j differs (exact, no carries across bytes)
+            uint32_t nz = (((x & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | x | dead[k]) & 0x80808080u;
+            if (edge) {
+#pragma unroll
+                for (int j = 0; j < 4; j++)
+                    if (d > lowp + j || p0 + j >= m) nz |= 0x80u << (8 * j);
+            }
+            const uint32_t c = (uint32_t)(256 - d);
+            int r = bnd ? 0 : R[k];
+            r = (nz & 0x80000000u) ? 0 : min(r + 1, F);
+            best3 = max(best3, ((uint32_t)r << 8) | c);
+            r = (nz & 0x00800000u) ? 0 : min(r + 1, F);
+            best2 = max(best2, ((uint32_t)r << 8) | c);
+            r = (nz & 0x00008000u) ? 0 : min(r + 1, F);
+            best1 = max(best1, ((uint32_t)r << 8) | c);
+            r = (nz & 0x00000080u) ? 0 : min(r + 1, F);
+            best0 = max(best0, ((uint32_t)r << 8) | c);
+            R[k] = r;
+        }
+        best0 = __reduce_max_sync(kFull, best0);
+        best1 = __reduce_max_sync(kFull, best1);
+        best2 = __reduce_max_sync(kFull, best2);
+        best3 = __reduce_max_sync(kFull, best3);
+        if (lane < 4 && p0 + lane < r1) {
+            const uint32_t b = lane == 0 ? best0 : lane == 1 ? best1 : lane == 2 ? best2 : best3;
+            ld[sk2(p0 + lane)] = b >= (3u << 8) ? (uint16_t)Memo<true>::match((int)(256 - (b & 0xFF)), (int)(b >> 8))
+                                                : Memo<true>::kLit;
+        }
+    };
+    int p0 = (r1 - 1) & ~3;
+    if (p0 + 4 > m) {  // the buffer's last, partial word
+        step(p0, true);
+        p0 -= 4;
+    }
+#pragma unroll 1
+    while (p0 >= r0) {
+        // straight-line steps down to the first W positions of p0's chunk
+        // (they always read bytes >= 0: p0 - d >= chunk start)
+        const int fe = max(r0, (p0 & ~smask) + ((W + 3) & ~3));
+#pragma unroll 1
+        for (; p0 >= fe; p0 -= 4) step(p0, false);
+#pragma unroll 1
+        for (; p0 >= r0 && (p0 & smask) < W; p0 -= 4) step(p0, true);
     }
 }
 
@@ -777,8 +858,15 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
         }
         pair_sync(bar);  // tab is dead from here on
         if (V2) {
-            // version 2: (L, D) of every position by the warp-cooperative search
-            v2_search_all(sm.cw, sm.a.u.w.ld, m, W, F, half, lane, smask);
+            // version 2: (L, D) of every position by the warp-cooperative search,
+            // on an unskewed little-endian copy of the chunk (+ zero tail)
+            uint32_t *U = sm.a.u.w.ucw;
+            for (int j = t64; j < kUcwWords; j += kWalkLanes) U[j] = j < kChunkMax / 4 ? sm.cw[j + (j >> 5)] : 0u;
+            pair_sync(bar);
+            if (W <= 128)
+                v2_search_all<4>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
+            else
+                v2_search_all<8>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
             pair_sync(bar);
         }
 
