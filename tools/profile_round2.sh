@@ -27,6 +27,19 @@ for cfg in c3_runs20_1g c2_csource_128m c4_random_1g c5_tarmix_64g; do
       -o gpurun_out/full_${cfg}_$TAG python bench.py --config $cfg --steps 1 --warmup 1 --no-cpu-baseline --no-e2e \
       --no-versions --no-decompress --no-other-configs > /dev/null 2>&1
 done
+for cfg in c2_csource_128m c3_runs20_1g c4_random_1g; do bash tools/dec_launch.sh $TAG $cfg > gpurun_out/declaunch_${cfg}_$TAG.txt 2>&1; done
+CULZSS_BENCH_NO_LIVE_PEAK=1 ncu --set full --clock-control none --import-source on -k regex:decode_kernel -s 1 -c 1 \
+    -o gpurun_out/full_decode_kernel_c3_$TAG python bench.py --config c3_runs20_1g --steps 1 --warmup 1 --no-cpu-baseline \
+    --no-e2e --no-versions --no-other-configs > /dev/null 2>&1
+CULZSS_BENCH_NO_LIVE_PEAK=1 ncu --set full --clock-control none --import-source on -k regex:literal_kernel -s 1 -c 1 \
+    -o gpurun_out/full_literal_kernel_c4_$TAG python bench.py --config c4_random_1g --steps 1 --warmup 1 --no-cpu-baseline \
+    --no-e2e --no-versions --no-other-configs > /dev/null 2>&1
+# version 2: the bench's versions leg launches the V2 instantiation (-s 1 skips its warm-up launch;
+# the filter matches the demangled name of the V2 instantiation only)
+CULZSS_BENCH_NO_LIVE_PEAK=1 ncu --set full --clock-control none --import-source on \
+    --kernel-name-base demangled -k 'regex:chunk_kernel<0, (0|false), (1|true)' -s 1 -c 1 \
+    -o gpurun_out/full_v2_c2_$TAG python bench.py --config c2_csource_128m --steps 1 --warmup 1 --no-cpu-baseline \
+    --no-e2e --no-decompress --no-other-configs > /dev/null 2>&1
 for k in walk_kernel decode_kernel; do
   CULZSS_BENCH_NO_LIVE_PEAK=1 ncu --set full --clock-control none --import-source on -k regex:$k -s 1 -c 1 \
       -o gpurun_out/full_${k}_c2_$TAG python bench.py --config c2_csource_128m --steps 1 --warmup 1 --no-cpu-baseline \

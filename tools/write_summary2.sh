@@ -52,16 +52,36 @@ print("## Fused chunk kernel (rows a1-a4), --set full\n")
 for cfg in ("c3_runs20_1g", "c2_csource_128m", "c4_random_1g", "c5_tarmix_64g"):
     run("tools/ncu_summary.py", "full", f"gpurun_out/full_{cfg}_{t}.ncu-rep", cfg)
 print("### Per-phase split (tools/ncu_lines.py: warp instructions / stall samples by source line range)\n")
-rng = ["78:218:helpers", "219:285:evalpos", "286:340:bndbuild", "341:431:machine1", "432:523:machine2",
-       "524:556:walkfix", "655:697:stage", "698:794:build", "795:875:mask", "876:921:fixup", "922:1030:emit",
-       "1031:1102:scan+write"]
+# phase line ranges from markers in the source (so they follow edits)
+src = open("paper_conf_cluster_ozsoys11_b200/csrc/lzss_chunk.cu").read().split("\n")
+def at(marker):
+    return next(i + 1 for i, l in enumerate(src) if marker in l)
+marks = [("// skewed byte index", "helpers"), ("__device__ uint32_t eval_pos", "evalpos"),
+         ("// Run-boundary mask of a warp", "bndbuild"), ("// Speculative greedy walk", "machine1"),
+         ("// ---- machine 2", "machine2"), ("// Re-walk from a corrected", "walkfix"),
+         ("// Version 2: the paper", "version2"), ("void pair_sync(int id)", "kernelhead"),
+         ("---------------- a1: stage", "stage"), ("---------------- a2 part 1", "build"),
+         ("---------------- a3: lazy", "mask"), ("const int spec_exit =", "fixup"),
+         ("---------------- a4: bit-pack", "emit"), ("exclusive scan of bit counts over the 64", "scan+write")]
+starts = [(at(m), name) for m, name in marks]
+rng = [f"{a}:{(starts[i + 1][0] - 1) if i + 1 < len(starts) else len(src)}:{name}" for i, (a, name) in enumerate(starts)]
 for cfg in ("c3_runs20_1g", "c2_csource_128m", "c5_tarmix_64g"):
     print(f"{cfg}:\n```")
     print(subprocess.run(["python", "tools/ncu_lines.py", f"gpurun_out/full_{cfg}_{t}.ncu-rep", "lzss_chunk.cu", *rng,
                           "--top", "10"], capture_output=True, text=True).stdout + "```\n")
-print("## Decoder (row a6), --set full, c2 stream\n")
+print("## Decoder (row a6), --set full\n")
 for k in ("walk_kernel", "decode_kernel"):
-    run("tools/ncu_summary.py", "full", f"gpurun_out/full_{k}_c2_{t}.ncu-rep", k)
+    run("tools/ncu_summary.py", "full", f"gpurun_out/full_{k}_c2_{t}.ncu-rep", k + " (c2 stream)")
+run("tools/ncu_summary.py", "full", f"gpurun_out/full_decode_kernel_c3_{t}.ncu-rep", "decode_kernel (c3 stream)")
+run("tools/ncu_summary.py", "full", f"gpurun_out/full_literal_kernel_c4_{t}.ncu-rep", "literal_kernel (c4 stream)")
+print("### Decoder launch lists per config (classify / literal / walk / decode, cold and serialised)\n")
+for cfg in ("c2_csource_128m", "c3_runs20_1g", "c4_random_1g"):
+    try:
+        print(f"{cfg}:\n```\n" + open(f"gpurun_out/declaunch_{cfg}_{t}.txt").read() + "```\n")
+    except Exception:
+        pass
+print("## Version 2 (the paper's all-position search), --set full, c2\n")
+run("tools/ncu_summary.py", "full", f"gpurun_out/full_v2_c2_{t}.ncu-rep", "chunk_kernel, params.version = 2")
 PY
 python - "$TAG" <<'PY'
 import csv, io, json, subprocess, sys
