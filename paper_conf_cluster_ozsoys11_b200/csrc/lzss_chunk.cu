@@ -574,7 +574,7 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
     const int M0 = ((m >> 1) + 3) & ~3;
     const int r0 = half ? M0 : 0, r1 = half ? m : M0;
     if (r0 >= r1) return;
-    int R[K];
+    uint32_t R[K];     // (R_d << 8) | (256 - d) at the last position swept
     uint32_t dead[K];  // 0x80808080: offset beyond W (never matches)
 #pragma unroll
     for (int k = 0; k < K; k++) {
@@ -595,7 +595,7 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
             }
             r = min(r, cap);
         }
-        R[k] = r;
+        R[k] = ((uint32_t)r << 8) | (uint32_t)(256 - d);
     }
     // One step: the 4 positions of word p0.  EDGE steps (the first W
     // positions of a chunk, where d > p - chunk start, and the buffer's last,
@@ -633,16 +633,18 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
                 for (int j = 0; j < 4; j++)
                     if (d > lowp + j || p0 + j >= m) nz |= 0x80u << (8 * j);
             }
-            const uint32_t c = (uint32_t)(256 - d);
-            int r = bnd ? 0 : R[k];
-            r = (nz & 0x80000000u) ? 0 : min(r + 1, F);
-            best3 = max(best3, ((uint32_t)r << 8) | c);
-            r = (nz & 0x00800000u) ? 0 : min(r + 1, F);
-            best2 = max(best2, ((uint32_t)r << 8) | c);
-            r = (nz & 0x00008000u) ? 0 : min(r + 1, F);
-            best1 = max(best1, ((uint32_t)r << 8) | c);
-            r = (nz & 0x00000080u) ? 0 : min(r + 1, F);
-            best0 = max(best0, ((uint32_t)r << 8) | c);
+            // the recurrence carried on the key (R << 8) | c itself: +256 per
+            // equal byte, capped at (F << 8) | c, back to c (R = 0) on a difference
+            const uint32_t c = (uint32_t)(256 - d), fk = ((uint32_t)F << 8) | c;
+            uint32_t r = bnd ? c : R[k];
+            r = (nz & 0x80000000u) ? c : min(r + 256u, fk);
+            best3 = max(best3, r);
+            r = (nz & 0x00800000u) ? c : min(r + 256u, fk);
+            best2 = max(best2, r);
+            r = (nz & 0x00008000u) ? c : min(r + 256u, fk);
+            best1 = max(best1, r);
+            r = (nz & 0x00000080u) ? c : min(r + 256u, fk);
+            best0 = max(best0, r);
             R[k] = r;
         }
         best0 = __reduce_max_sync(kFull, best0);

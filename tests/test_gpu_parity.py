@@ -221,6 +221,61 @@ def test_gpu_decoder_rejects_corrupt(env):
             assert gst in (culzss.ERR_CORRUPT, culzss.ERR_UNSUPPORTED)
 
 
+def test_gpu_decoder_incompressible_chunks(env):
+    """Chunks of size ceil(9m/8) (PAPER.md:1@6743 §II.A.2 decoding; such a chunk
+    holds only literals in a valid stream) skip the walk and decode in the literal kernel, which
+    must check every flag bit and the pad bits exactly as the oracle decoder does."""
+    torch, culzss = env
+    S = 4096
+    for n in (3 * S + 1001, 2 * S, 17, 5 * S + 8):
+        x = datagen.generate("random", n, seed=n)
+        s = O.compress(x)
+        C = (n + S - 1) // S
+        sizes = np.frombuffer(s[32:32 + 4 * C], "<u4")
+        ms = [min(S, n - c * S) for c in range(C)]
+        assert all(int(sz) == (9 * m + 7) // 8 for sz, m in zip(sizes, ms)), "random chunks are all-literal"
+        y = culzss.decompress(dev(torch, np.frombuffer(s, np.uint8)))
+        assert y.cpu().numpy().tobytes() == x.tobytes(), n
+        base = 32 + 4 * C
+        off = base + int(sizes[:C - 1].sum())  # the last chunk's payload
+        m = ms[-1]
+        for j in (0, 1, m // 2, m - 1):  # a literal's flag bit set: the oracle and the GPU reject
+            b = bytearray(s)
+            bit = 9 * j
+            b[off + bit // 8] |= 0x80 >> (bit % 8)
+            assert O.decompress_status(bytes(b))[0] == O.ERR_CORRUPT
+            st, _ = culzss.decompress_status(dev(torch, np.frombuffer(bytes(b), np.uint8)))
+            assert st == culzss.ERR_CORRUPT, (n, j)
+        pad = 8 * int(sizes[-1]) - 9 * m
+        if pad:  # a nonzero pad bit
+            b = bytearray(s)
+            b[off + int(sizes[-1]) - 1] |= 1
+            assert O.decompress_status(bytes(b))[0] == O.ERR_CORRUPT
+            st, _ = culzss.decompress_status(dev(torch, np.frombuffer(bytes(b), np.uint8)))
+            assert st == culzss.ERR_CORRUPT, n
+
+
+def test_gpu_decoder_mutations_mixed(env):
+    """Random mutations of a stream mixing incompressible, text and run chunks (the classify /
+    literal / walk / decode kernels all see malformed input): CORRUPT, or the oracle's output."""
+    torch, culzss = env
+    rng = np.random.default_rng(11)
+    x = np.concatenate([datagen.generate("random", 2 * 4096 + 300, seed=1), datagen.generate("english", 9000, seed=2),
+                        datagen.generate("runs20", 5000, seed=3), datagen.generate("random", 4096, seed=4)])
+    base = bytearray(O.compress(x))
+    for _ in range(200):
+        s = bytearray(base)
+        for _ in range(int(rng.integers(1, 4))):
+            i = int(rng.integers(32, len(s)))
+            s[i] ^= int(rng.integers(1, 256))
+        ost, oout = O.decompress_status(bytes(s))
+        gst, gout = culzss.decompress_status(dev(torch, np.frombuffer(bytes(s), np.uint8)))
+        if ost == O.OK:
+            assert gst == culzss.OK and gout.cpu().numpy().tobytes() == oout
+        else:
+            assert gst in (culzss.ERR_CORRUPT, culzss.ERR_UNSUPPORTED)
+
+
 def test_unaligned_input_and_output(env):
     torch, culzss = env
     x = datagen.generate("csource", 100000, seed=8)
