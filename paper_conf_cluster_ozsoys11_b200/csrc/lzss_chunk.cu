@@ -575,11 +575,11 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
     const int r0 = half ? M0 : 0, r1 = half ? m : M0;
     if (r0 >= r1) return;
     uint32_t R[K];     // (R_d << 8) | (256 - d) at the last position swept
-    uint32_t dead[K];  // 0x80808080: offset beyond W (never matches)
+    uint32_t dead[K];  // all ones: offset beyond W (never matches)
 #pragma unroll
     for (int k = 0; k < K; k++) {
         const int d = lane + 1 + 32 * k;
-        dead[k] = d <= W ? 0u : 0x80808080u;
+        dead[k] = d <= W ? 0u : 0xFFFFFFFFu;
         // the run at r1 (the carry into the sweep): 0 at the chunk end or at a
         // packed chunk boundary, else measured directly
         int r = 0;
@@ -610,8 +610,8 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
         const uint32_t P = U[p0 >> 2];
         const int lowp = p0 & smask;               // position of p0 in its chunk
         const bool bnd = ((p0 + 4) & smask) == 0;  // a chunk ends after this word: no carry
-        uint32_t best0 = 0, best1 = 0, best2 = 0, best3 = 0;
         const unsigned char *qa = Ub + (p0 - c4);
+        uint32_t rk[K][4];  // key (R << 8) | c of positions p0 + j, per offset
 #pragma unroll
         for (int k = 0; k < K; k++) {
             const int d = lane + 1 + 32 * k;
@@ -625,28 +625,39 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
                 const int q = p0 - d;
                 Q = q >= 0 ? v2_bytes4(U, q) : v2_bytes4(U, 0) << (8 * min(-q, 3));
             }
-            const uint32_t x = P ^ Q;
-            // bit 7 of byte j set iff byte j differs (exact, no carries across bytes)
-            uint32_t nz = (((x & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | x | dead[k]) & 0x80808080u;
+            // byte j of x is 0 iff positions p0 + j and p0 + j - d hold equal bytes
+            // (a dead offset, d > W, never matches)
+            uint32_t x = (P ^ Q) | dead[k];
             if (edge) {
 #pragma unroll
                 for (int j = 0; j < 4; j++)
-                    if (d > lowp + j || p0 + j >= m) nz |= 0x80u << (8 * j);
+                    if (d > lowp + j || p0 + j >= m) x |= 0xFFu << (8 * j);
             }
             // the recurrence carried on the key (R << 8) | c itself: +256 per
             // equal byte, capped at (F << 8) | c, back to c (R = 0) on a difference
             const uint32_t c = (uint32_t)(256 - d), fk = ((uint32_t)F << 8) | c;
             uint32_t r = bnd ? c : R[k];
-            r = (nz & 0x80000000u) ? c : min(r + 256u, fk);
-            best3 = max(best3, r);
-            r = (nz & 0x00800000u) ? c : min(r + 256u, fk);
-            best2 = max(best2, r);
-            r = (nz & 0x00008000u) ? c : min(r + 256u, fk);
-            best1 = max(best1, r);
-            r = (nz & 0x00000080u) ? c : min(r + 256u, fk);
-            best0 = max(best0, r);
+            r = (x & 0xFF000000u) ? c : min(r + 256u, fk);
+            rk[k][3] = r;
+            r = (x & 0x00FF0000u) ? c : min(r + 256u, fk);
+            rk[k][2] = r;
+            r = (x & 0x0000FF00u) ? c : min(r + 256u, fk);
+            rk[k][1] = r;
+            r = (x & 0x000000FFu) ? c : min(r + 256u, fk);
+            rk[k][0] = r;
             R[k] = r;
         }
+        // the lane's best key per position: three-input maxima over its offsets
+        uint32_t bj[4];
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            uint32_t b = rk[0][j];
+#pragma unroll
+            for (int k = 1; k < K; k += 2)
+                b = k + 1 < K ? __vimax3_u32(b, rk[k][j], rk[k + 1][j]) : max(b, rk[k][j]);
+            bj[j] = b;
+        }
+        uint32_t best0 = bj[0], best1 = bj[1], best2 = bj[2], best3 = bj[3];
         best0 = __reduce_max_sync(kFull, best0);
         best1 = __reduce_max_sync(kFull, best1);
         best2 = __reduce_max_sync(kFull, best2);
