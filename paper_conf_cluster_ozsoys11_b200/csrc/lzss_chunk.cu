@@ -606,6 +606,13 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
     const int c4 = (lane + 4) & ~3;
     const uint32_t shq = 8u * (uint32_t)((-(lane + 1)) & 3);
     const unsigned char *Ub = reinterpret_cast<const unsigned char *>(U);
+    uint32_t mine = 0;  // the argmax key of position (block base) + lane
+    auto flush = [&](int blk) {  // positions blk .. blk + 31 (those of this warp)
+        const int p = blk + lane;
+        if (p >= r0 && p < r1)
+            ld[sk2(p)] = mine >= (3u << 8) ? (uint16_t)Memo<true>::match((int)(256 - (mine & 0xFF)), (int)(mine >> 8))
+                                           : Memo<true>::kLit;
+    };
     auto step = [&](int p0, bool edge) {
         const uint32_t P = U[p0 >> 2];
         const int lowp = p0 & smask;               // position of p0 in its chunk
@@ -662,11 +669,11 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
         best1 = __reduce_max_sync(kFull, best1);
         best2 = __reduce_max_sync(kFull, best2);
         best3 = __reduce_max_sync(kFull, best3);
-        if (lane < 4 && p0 + lane < r1) {
-            const uint32_t b = lane == 0 ? best0 : lane == 1 ? best1 : lane == 2 ? best2 : best3;
-            ld[sk2(p0 + lane)] = b >= (3u << 8) ? (uint16_t)Memo<true>::match((int)(256 - (b & 0xFF)), (int)(b >> 8))
-                                                : Memo<true>::kLit;
-        }
+        // lane t keeps the key of position (p0 & ~31) + t; the warp stores a
+        // block of 32 positions once its lowest word is done
+        const int t = lane - (p0 & 31);
+        mine = t == 0 ? best0 : t == 1 ? best1 : t == 2 ? best2 : t == 3 ? best3 : mine;
+        if ((p0 & 31) == 0) flush(p0);
     };
     int p0 = (r1 - 1) & ~3;
     if (p0 + 4 > m) {  // the buffer's last, partial word
@@ -683,6 +690,7 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
 #pragma unroll 1
         for (; p0 >= r0 && (p0 & smask) < W; p0 -= 4) step(p0, true);
     }
+    if (r0 & 31) flush(r0 & ~31);  // the last, partial block
 }
 
 // greedy parse over a fully evaluated token table: jump from p to the end of
