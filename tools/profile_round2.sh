@@ -35,9 +35,9 @@ CULZSS_BENCH_NO_LIVE_PEAK=1 ncu --set full --clock-control none --import-source 
     -o gpurun_out/full_literal_kernel_c4_$TAG python bench.py --config c4_random_1g --steps 1 --warmup 1 --no-cpu-baseline \
     --no-e2e --no-versions --no-other-configs > /dev/null 2>&1
 # version 2: the bench's versions leg launches the V2 instantiation (-s 1 skips its warm-up launch;
-# the filter matches the demangled name of the V2 instantiation only)
+# the filter matches the mangled name of the V2 instantiation only)
 CULZSS_BENCH_NO_LIVE_PEAK=1 ncu --set full --clock-control none --import-source on \
-    --kernel-name-base demangled -k 'regex:chunk_kernel<0, (0|false), (1|true)' -s 1 -c 1 \
+    --kernel-name-base mangled -k 'regex:chunk_kernelILi0ELb0ELb1ELb0ELb0E' -s 1 -c 1 \
     -o gpurun_out/full_v2_c2_$TAG python bench.py --config c2_csource_128m --steps 1 --warmup 1 --no-cpu-baseline \
     --no-e2e --no-decompress --no-other-configs > /dev/null 2>&1
 for k in walk_kernel decode_kernel; do
