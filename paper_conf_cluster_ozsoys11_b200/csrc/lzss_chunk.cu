@@ -616,7 +616,6 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
     auto step = [&](int p0, bool edge) {
         const uint32_t P = U[p0 >> 2];
         const int lowp = p0 & smask;               // position of p0 in its chunk
-        const bool bnd = ((p0 + 4) & smask) == 0;  // a chunk ends after this word: no carry
         const unsigned char *qa = Ub + (p0 - c4);
         uint32_t rk[K][4];  // key (R << 8) | c of positions p0 + j, per offset
 #pragma unroll
@@ -643,7 +642,7 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
             // the recurrence carried on the key (R << 8) | c itself: +256 per
             // equal byte, capped at (F << 8) | c, back to c (R = 0) on a difference
             const uint32_t c = (uint32_t)(256 - d), fk = ((uint32_t)F << 8) | c;
-            uint32_t r = bnd ? c : R[k];
+            uint32_t r = R[k];
             r = (x & 0xFF000000u) ? c : min(r + 256u, fk);
             rk[k][3] = r;
             r = (x & 0x00FF0000u) ? c : min(r + 256u, fk);
@@ -671,8 +670,10 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
         best3 = __reduce_max_sync(kFull, best3);
         // lane t keeps the key of position (p0 & ~31) + t; the warp stores a
         // block of 32 positions once its lowest word is done
-        const int t = lane - (p0 & 31);
-        mine = t == 0 ? best0 : t == 1 ? best1 : t == 2 ? best2 : t == 3 ? best3 : mine;
+        const unsigned t = (unsigned)(lane - (p0 & 31));
+        const uint32_t s01 = (t & 1) ? best1 : best0, s23 = (t & 1) ? best3 : best2;
+        const uint32_t sv = (t & 2) ? s23 : s01;
+        mine = t < 4 ? sv : mine;
         if ((p0 & 31) == 0) flush(p0);
     };
     int p0 = (r1 - 1) & ~3;
@@ -682,6 +683,10 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
     }
 #pragma unroll 1
     while (p0 >= r0) {
+        if (((p0 + 4) & smask) == 0) {  // a chunk ends above this word: no carry into it
+#pragma unroll
+            for (int k = 0; k < K; k++) R[k] = (uint32_t)(256 - (lane + 1 + 32 * k));
+        }
         // straight-line steps down to the first W positions of p0's chunk
         // (they always read bytes >= 0: p0 - d >= chunk start)
         const int fe = max(r0, (p0 & ~smask) + ((W + 3) & ~3));
