@@ -567,7 +567,18 @@ __device__ __forceinline__ uint32_t v2_bytes4(const uint32_t *__restrict__ U, in
     return __funnelshift_r(U[a], U[a + 1], (uint32_t)x << 3);  // the shift is taken mod 32
 }
 
-template <int K>
+// prmt with the selector's sign-replicate bit honoured (__byte_perm masks it)
+__device__ __forceinline__ uint32_t prmt_sx(uint32_t a, uint32_t b, uint32_t sel) {
+    uint32_t r;
+    asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
+    return r;
+}
+
+// P16 (K = 4, F <= 254): two offsets' keys per register as 16-bit halves,
+// updated by the 16x2 forms (VIADDMNMX.U16x2, VIMNMX.U16x2); a position's
+// two "differs" half-masks come from one sign-replicating byte permute of the
+// two offsets' per-byte difference bits.
+template <int K, bool P16>
 __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restrict__ ld, int m, int W, int F,
                               int half, int lane, int smask) {
     // warp 0: positions [0, M0), warp 1: [M0, m); M0 is a word boundary
@@ -597,6 +608,14 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
         }
         R[k] = ((uint32_t)r << 8) | (uint32_t)(256 - d);
     }
+    // P16: offsets 2q (low half) and 2q + 1 (high half) share register q
+    uint32_t R2[K / 2], c2[K / 2], fk2[K / 2];
+#pragma unroll
+    for (int q = 0; q < K / 2; q++) {
+        c2[q] = (uint32_t)(256 - (lane + 1 + 64 * q)) | ((uint32_t)(256 - (lane + 33 + 64 * q)) << 16);
+        fk2[q] = c2[q] | ((uint32_t)F << 8) | ((uint32_t)F << 24);
+        R2[q] = (R[2 * q] & 0xFFFFu) | (R[2 * q + 1] << 16);
+    }
     // One step: the 4 positions of word p0.  EDGE steps (the first W
     // positions of a chunk, where d > p - chunk start, and the buffer's last,
     // partial word) mask the invalid pairs; the others are straight-line: for
@@ -609,15 +628,17 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
     uint32_t mine = 0;  // the argmax key of position (block base) + lane
     auto flush = [&](int blk) {  // positions blk .. blk + 31 (those of this warp)
         const int p = blk + lane;
+        const uint32_t key = P16 ? (mine & 0xFFFFu) : mine;
         if (p >= r0 && p < r1)
-            ld[sk2(p)] = mine >= (3u << 8) ? (uint16_t)Memo<true>::match((int)(256 - (mine & 0xFF)), (int)(mine >> 8))
-                                           : Memo<true>::kLit;
+            ld[sk2(p)] = key >= (3u << 8) ? (uint16_t)Memo<true>::match((int)(256 - (key & 0xFF)), (int)(key >> 8))
+                                          : Memo<true>::kLit;
     };
     auto step = [&](int p0, bool edge) {
         const uint32_t P = U[p0 >> 2];
         const int lowp = p0 & smask;               // position of p0 in its chunk
         const unsigned char *qa = Ub + (p0 - c4);
         uint32_t rk[K][4];  // key (R << 8) | c of positions p0 + j, per offset
+        uint32_t nzv[K];    // P16: per-byte difference bits, per offset
 #pragma unroll
         for (int k = 0; k < K; k++) {
             const int d = lane + 1 + 32 * k;
@@ -639,29 +660,59 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
                 for (int j = 0; j < 4; j++)
                     if (d > lowp + j || p0 + j >= m) x |= 0xFFu << (8 * j);
             }
-            // the recurrence carried on the key (R << 8) | c itself: +256 per
-            // equal byte, capped at (F << 8) | c, back to c (R = 0) on a difference
-            const uint32_t c = (uint32_t)(256 - d), fk = ((uint32_t)F << 8) | c;
-            uint32_t r = R[k];
-            r = (x & 0xFF000000u) ? c : min(r + 256u, fk);
-            rk[k][3] = r;
-            r = (x & 0x00FF0000u) ? c : min(r + 256u, fk);
-            rk[k][2] = r;
-            r = (x & 0x0000FF00u) ? c : min(r + 256u, fk);
-            rk[k][1] = r;
-            r = (x & 0x000000FFu) ? c : min(r + 256u, fk);
-            rk[k][0] = r;
-            R[k] = r;
+            if constexpr (P16) {
+                nzv[k] = ((x & 0x7F7F7F7Fu) + 0x7F7F7F7Fu) | x;  // bit 7 of byte j: differs
+            } else {
+                // the recurrence carried on the key (R << 8) | c itself: +256 per
+                // equal byte, capped at (F << 8) | c, back to c (R = 0) on a difference
+                const uint32_t c = (uint32_t)(256 - d), fk = ((uint32_t)F << 8) | c;
+                uint32_t r = R[k];
+                r = (x & 0xFF000000u) ? c : min(r + 256u, fk);
+                rk[k][3] = r;
+                r = (x & 0x00FF0000u) ? c : min(r + 256u, fk);
+                rk[k][2] = r;
+                r = (x & 0x0000FF00u) ? c : min(r + 256u, fk);
+                rk[k][1] = r;
+                r = (x & 0x000000FFu) ? c : min(r + 256u, fk);
+                rk[k][0] = r;
+                R[k] = r;
+            }
         }
-        // the lane's best key per position: three-input maxima over its offsets
         uint32_t bj[4];
+        if constexpr (P16) {
+            uint32_t rk2[K / 2][4];
 #pragma unroll
-        for (int j = 0; j < 4; j++) {
-            uint32_t b = rk[0][j];
+            for (int q = 0; q < K / 2; q++) {
+                uint32_t r = R2[q];
 #pragma unroll
-            for (int k = 1; k < K; k += 2)
-                b = k + 1 < K ? __vimax3_u32(b, rk[k][j], rk[k + 1][j]) : max(b, rk[k][j]);
-            bj[j] = b;
+                for (int j = 3; j >= 0; j--) {
+                    // halves 0xFFFF where position p0 + j differs for offset 2q / 2q + 1
+                    const uint32_t msk = prmt_sx(nzv[2 * q], nzv[2 * q + 1],
+                                                 (uint32_t)((8 + j) | ((8 + j) << 4) | ((12 + j) << 8) | ((12 + j) << 12)));
+                    r = __viaddmin_u16x2(r, 0x01000100u, fk2[q]);
+                    r = (r & ~msk) | (c2[q] & msk);
+                    rk2[q][j] = r;
+                }
+                R2[q] = r;
+            }
+#pragma unroll
+            for (int j = 0; j < 4; j++) {
+                uint32_t mm = rk2[0][j];
+#pragma unroll
+                for (int q = 1; q < K / 2; q++) mm = __vmaxu2(mm, rk2[q][j]);
+                bj[j] = __vmaxu2(mm, __byte_perm(mm, 0, 0x1032));  // the larger key in both halves
+            }
+        } else {
+            // the lane's best key per position: three-input maxima over its offsets
+    #pragma unroll
+            for (int j = 0; j < 4; j++) {
+                uint32_t b = rk[0][j];
+    #pragma unroll
+                for (int k = 1; k < K; k += 2)
+                    b = k + 1 < K ? __vimax3_u32(b, rk[k][j], rk[k + 1][j]) : max(b, rk[k][j]);
+                bj[j] = b;
+            }
+
         }
         uint32_t best0 = bj[0], best1 = bj[1], best2 = bj[2], best3 = bj[3];
         best0 = __reduce_max_sync(kFull, best0);
@@ -686,6 +737,8 @@ __device__ void v2_search_all(const uint32_t *__restrict__ U, uint16_t *__restri
         if (((p0 + 4) & smask) == 0) {  // a chunk ends above this word: no carry into it
 #pragma unroll
             for (int k = 0; k < K; k++) R[k] = (uint32_t)(256 - (lane + 1 + 32 * k));
+#pragma unroll
+            for (int q = 0; q < K / 2; q++) R2[q] = c2[q];
         }
         // straight-line steps down to the first W positions of p0's chunk
         // (they always read bytes >= 0: p0 - d >= chunk start)
@@ -889,10 +942,12 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
             uint32_t *U = sm.a.u.w.ucw;
             for (int j = t64; j < kUcwWords; j += kWalkLanes) U[j] = j < kChunkMax / 4 ? sm.cw[j + (j >> 5)] : 0u;
             pair_sync(bar);
-            if (W <= 128)
-                v2_search_all<4>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
+            if (W <= 128 && F <= 254)
+                v2_search_all<4, true>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
+            else if (W <= 128)
+                v2_search_all<4, false>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
             else
-                v2_search_all<8>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
+                v2_search_all<8, false>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
             pair_sync(bar);
         }
 

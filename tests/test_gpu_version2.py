@@ -49,7 +49,11 @@ def test_v2_stream_bit_exact_generators(env, kind):
 
 @pytest.mark.parametrize("S,W,F", [(4096, 1, 3), (4096, 16, 18), (4096, 64, 200), (4096, 255, 258),
                                    (4096, 129, 129), (1, 128, 128), (100, 7, 9), (1000, 128, 128),
-                                   (129, 3, 5)])
+                                   (129, 3, 5),
+                                   # the sweep's instantiations: 16-bit keys (W <= 128, F <= 254) and
+                                   # 32-bit keys (F >= 255) at their border, packed chunks
+                                   (4096, 128, 254), (4096, 128, 255), (4096, 100, 258), (256, 128, 254),
+                                   (512, 64, 258)])
 def test_v2_stream_params_variants(env, S, W, F):
     for kind in ("english", "runs20", "period20", "binary"):
         if kind == "binary":
