@@ -574,7 +574,7 @@ __device__ __forceinline__ uint32_t prmt_sx(uint32_t a, uint32_t b, uint32_t sel
     return r;
 }
 
-// P16 (K = 4, F <= 254): two offsets' keys per register as 16-bit halves,
+// P16 (F <= 254): two offsets' keys per register as 16-bit halves,
 // updated by the 16x2 forms (VIADDMNMX.U16x2, VIMNMX.U16x2); a position's
 // two "differs" half-masks come from one sign-replicating byte permute of the
 // two offsets' per-byte difference bits.
@@ -942,10 +942,13 @@ chunk_kernel(const uint8_t *__restrict__ in, uint64_t n, Geometry g, uint8_t *__
             uint32_t *U = sm.a.u.w.ucw;
             for (int j = t64; j < kUcwWords; j += kWalkLanes) U[j] = j < kChunkMax / 4 ? sm.cw[j + (j >> 5)] : 0u;
             pair_sync(bar);
+            // 16-bit keys whenever (R << 8) | (256 - d) + 256 fits them: F <= 254
             if (W <= 128 && F <= 254)
                 v2_search_all<4, true>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
             else if (W <= 128)
                 v2_search_all<4, false>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
+            else if (F <= 254)
+                v2_search_all<8, true>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
             else
                 v2_search_all<8, false>(U, sm.a.u.w.ld, m, W, F, half, lane, smask);
             pair_sync(bar);

@@ -53,7 +53,7 @@ def test_v2_stream_bit_exact_generators(env, kind):
                                    # the sweep's instantiations: 16-bit keys (W <= 128, F <= 254) and
                                    # 32-bit keys (F >= 255) at their border, packed chunks
                                    (4096, 128, 254), (4096, 128, 255), (4096, 100, 258), (256, 128, 254),
-                                   (512, 64, 258)])
+                                   (512, 64, 258), (4096, 255, 254), (4096, 200, 100), (2048, 255, 128)])
 def test_v2_stream_params_variants(env, S, W, F):
     for kind in ("english", "runs20", "period20", "binary"):
         if kind == "binary":
